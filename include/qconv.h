@@ -1,0 +1,170 @@
+/*
+ * qconv.h -- C ABI of the B200 (sm_100a) 4/8-bit quantized convolution library
+ * (libqconv.so, built from paper_conf_icpp_hanhyylhgwwlq20_b200/csrc).
+ *
+ * The hot path of Han, Hu et al., "Extremely Low-bit Convolution Optimization
+ * for Quantized Neural Network on Modern Computer Architectures" (ICPP'20),
+ * section 4: quantization, implicit-GEMM convolution on tensor cores
+ * (Alg.2) with bias + re-quantization fused into the
+ * epilogue (P:L223 l.15) and ReLU folded into the truncation range
+ * (P:L265).  "P:Lnnn" = line nnn of the paper text; "Zn"/"R1" are
+ * the readings listed in DESIGN.md section 3.
+ *
+ * Conventions for every entry point
+ *  - Plain pointers and sizes only.  "device" pointers are CUDA device
+ *    allocations owned by the caller; "host" pointers are host memory owned by
+ *    the caller.  The library never allocates device memory and never frees a
+ *    caller buffer.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  Device work is enqueued asynchronously on it; the call returns
+ *    after enqueueing.  Argument errors are detected on the host and returned
+ *    synchronously before anything is enqueued; a failed launch returns
+ *    QC_ERR_CUDA (qconv_last_cuda_error() gives the CUDA error code).
+ *  - No call throws; all calls are reentrant and thread-safe (the only global
+ *    state is a lazily resolved driver entry point).
+ *  - Layouts: activations NHWC (C contiguous), weights KRSC (R*S*C
+ *    contiguous per output channel), outputs NHWC [N,P,Q,K].  4-bit tensors
+ *    pack two elements per byte, element 2j in the low nibble of byte j of the
+ *    row (reading Z7); signed 4-bit values are two's complement nibbles.
+ *  - P = (H + 2*pad_h - dil_h*(R-1) - 1)/stride_h + 1, Q likewise.
+ */
+#ifndef QCONV_H_
+#define QCONV_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    QC_OK = 0,
+    QC_ERR_INVALID_ARG = 1,    /* malformed shape / dtype / range / NULL pointer */
+    QC_ERR_UNSUPPORTED = 2,    /* well-formed but outside what the GPU path implements */
+    QC_ERR_OVERFLOW_RISK = 3,  /* int32 accumulation could overflow for this shape/dtype */
+    QC_ERR_MISALIGNED = 4,     /* a device pointer is not 16-byte aligned */
+    QC_ERR_WORKSPACE = 5,      /* workspace missing or smaller than qconv2d_workspace_size */
+    QC_ERR_CUDA = 6            /* a CUDA driver/runtime call failed */
+} qc_status;
+
+typedef enum { QC_U4 = 0, QC_S4 = 1, QC_U8 = 2, QC_S8 = 3, QC_S32 = 4 } qc_dtype;
+typedef enum { QC_F32 = 0, QC_BF16 = 1 } qc_ftype;
+
+/*
+ * qconv_quantize_pack -- quantization step of the QNN layer sequence,
+ * reading Z4: for every element, q = clamp(rne(x * fl32(1/scale)) + zero_point,
+ * qmin(yt), qmax(yt)), computed as one IEEE fp32 multiply then round-to-
+ * nearest-even (matches torch.quantize_per_tensor); NaN -> zero_point.
+ *   x          device, [npix, c] fp32 or bf16 (xt), npix = N*H*W
+ *   y          device, [npix, c_pad] packed yt in {U4,S4,U8,S8}; channels
+ *              c..c_pad-1 are written with zero_point (channel padding)
+ *   scale      > 0 and finite; zero_point inside the yt range
+ * Errors: INVALID_ARG (npix < 0, c < 1, c_pad < c, 4-bit with odd c_pad, bad
+ * scale/zero point/dtype, NULL), MISALIGNED (x or y not 16-byte aligned).
+ */
+qc_status qconv_quantize_pack(const void *x, qc_ftype xt, int64_t npix, int32_t c,
+                              int32_t c_pad, float scale, int32_t zero_point, qc_dtype yt,
+                              void *y, void *stream);
+
+/*
+ * qconv_requant_params -- host only, synchronous, deterministic (reading R1;
+ * the paper only says "re-quantize").  For k output channels:
+ *   M_k = fl64(fl64(in_scale) * fl64(w_scale[k])) / fl64(out_scale);
+ *   (f, e) = frexp(M_k); m = round-half-up(f * 2^31); if m == 2^31 {m = 2^30; e++}
+ *   multiplier[k] = m in [2^30, 2^31), shift[k] = 31 - e in [1, 62];
+ *   M_k == 0 gives (0, 31).
+ *   w_scale, multiplier, shift: host arrays of length k.
+ * Errors: INVALID_ARG (non-positive / non-finite scales, k < 1, NULL, or a
+ * shift outside [1, 62]).
+ */
+qc_status qconv_requant_params(float in_scale, const float *w_scale, float out_scale,
+                               int32_t k, int32_t *multiplier, int32_t *shift);
+
+/* Convolution descriptor (host struct, read during the call only). */
+typedef struct {
+    int32_t n, h, w, c, k, r, s;          /* X: [n,h,w,c] NHWC; W: [k,r,s,c] KRSC */
+    int32_t stride_h, stride_w;           /* 1..8 */
+    int32_t pad_h, pad_w;                 /* >= 0 (zero padding = real zero, Z2) */
+    int32_t dil_h, dil_w;                 /* >= 1 */
+    qc_dtype x_t, w_t, y_t;               /* x_t, w_t in {U4,S4,U8,S8}, same bit width;
+                                             y_t in {U4,S4,U8,S8,S32} */
+    int32_t x_zero;                       /* per-tensor activation zero point (Z1) */
+    int32_t w_prepared;                   /* 1: `w` is the output of qconv_prepare_weights */
+    int32_t y_zero;                       /* output zero point (ignored for S32) */
+    int32_t clamp_lo, clamp_hi;           /* truncation range inside the y_t range; ReLU:
+                                             clamp_lo = max(qmin, y_zero) (Z5);
+                                             ignored for S32 */
+} qconv_desc;
+
+/*
+ * qconv_prepare_weights -- once-per-layer weight preparation (the paper's
+ * "pre-processing"): KRSC weights of dtype d->w_t are widened to the
+ * kernel's operand layout, int8 KRSC (4-bit codes sign/zero-extended, since
+ * sm_100 tensor cores have no 4-bit integer MMA).  Output bytes:
+ * qconv_prepared_weight_bytes(d) = k*r*s*c.  8-bit weights are copied.
+ *   w       device, packed KRSC (d->w_t)
+ *   w_prep  device, >= qconv_prepared_weight_bytes(d) bytes
+ * Errors: INVALID_ARG, MISALIGNED, CUDA.
+ */
+size_t qconv_prepared_weight_bytes(const qconv_desc *d);
+qc_status qconv_prepare_weights(const qconv_desc *d, const void *w, void *w_prep, void *stream);
+
+/*
+ * qconv2d_workspace_size -- device workspace bytes qconv2d_forward needs for
+ * this descriptor: 0 unless x_zero != 0 (zero-point border table,
+ * k*(r+1)*(s+1) int32) or 4-bit weights are passed unprepared (w_prepared = 0:
+ * room for the widened copy).  Returns 0 for an invalid descriptor.
+ */
+size_t qconv2d_workspace_size(const qconv_desc *d);
+
+/*
+ * qconv2d_forward -- y = requant(conv(x - x_zero, w) + bias) (Alg.2).
+ * Per output (n,p,q,k), with acc = sum over in-bounds taps (r,s) and c of
+ * (x[n, p*sh-ph+r*dh, q*sw-pw+s*dw, c] - x_zero) * w[k,r,s,c] + bias[k]:
+ *   y_t == S32 : y = acc
+ *   otherwise  : t = floor((acc * multiplier[k] + 2^(shift[k]-1)) / 2^shift[k])
+ *                y = min(clamp_hi, max(clamp_lo, t + y_zero))     (Z3, Z5)
+ * Contract (the paper's 32-bit accumulator): |acc| < 2^31 for
+ * every output.  The host checks the dtype-range bound
+ * r*s*c*max|x-x_zero|*max|w| < 2^31 (else OVERFLOW_RISK); keeping acc + bias
+ * inside int32 is the caller's duty (bias is device data and is not read).
+ *   x          device, packed NHWC (d->x_t)
+ *   w          device, packed KRSC (d->w_t) or prepared (d->w_prepared = 1)
+ *   bias       device int32 [k] or NULL (= 0)
+ *   multiplier, shift   device int32 [k]; may be NULL only for y_t == S32
+ *   y          device, NHWC [n,p,q,k] packed y_t
+ *   workspace  device, >= qconv2d_workspace_size(d) bytes (NULL if 0)
+ * Errors: INVALID_ARG, UNSUPPORTED (mixed bit widths; c not a multiple of 32;
+ * 4-bit y_t with odd k; pad/dilation beyond the TMA im2col corner range;
+ * stride > 8), OVERFLOW_RISK, MISALIGNED, WORKSPACE, CUDA.
+ */
+qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w,
+                          const int32_t *bias, const int32_t *multiplier, const int32_t *shift,
+                          void *y, void *workspace, size_t ws_bytes, void *stream);
+
+/* Human-readable status; static storage, never NULL. */
+const char *qconv_status_string(qc_status s);
+
+/* CUDA error code (cudaError_t as int) of the last QC_ERR_CUDA on this thread. */
+int qconv_last_cuda_error(void);
+
+/* Library version (major*10000 + minor*100 + patch). */
+int qconv_version(void);
+
+/*
+ * Diagnostics (used by the parity tests, not on the hot path):
+ * qconv_debug_im2col_tile loads one 128-pixel im2col tile of x for GEMM row
+ * m0, filter tap (r, s) and channel byte offset c_byte (box = box_bytes bytes
+ * per pixel) with the same TMA descriptor construction as qconv2d_forward but
+ * without swizzle, and writes it to `out` (device, 128*box_bytes bytes).
+ */
+qc_status qconv_debug_im2col_tile(const qconv_desc *d, const void *x, int64_t m0, int32_t r,
+                                  int32_t s, int32_t c_byte, int32_t box_bytes, void *out,
+                                  void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* QCONV_H_ */

@@ -1,0 +1,250 @@
+"""B200-native 4/8-bit quantized convolution (Han, Hu et al., ICPP'20, section 4).
+
+Thin Python binding over the C ABI of libqconv.so (include/qconv.h): argument
+marshalling only -- every step of the hot path (quantize+pack, implicit-GEMM
+convolution on tcgen05 tensor cores, fused bias/re-quantization/ReLU/packing)
+runs in the library's CUDA kernels.  PyTorch is used for device memory and
+streams.  There is no CPU fallback: if libqconv.so is missing, importing
+this package raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+from typing import Optional, Sequence, Tuple
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_PKG, "libqconv.so")
+
+QC_U4, QC_S4, QC_U8, QC_S8, QC_S32 = 0, 1, 2, 3, 4
+QC_F32, QC_BF16 = 0, 1
+_BITS = {QC_U4: 4, QC_S4: 4, QC_U8: 8, QC_S8: 8, QC_S32: 32}
+_RANGE = {QC_U4: (0, 15), QC_S4: (-8, 7), QC_U8: (0, 255), QC_S8: (-128, 127),
+          QC_S32: (-(2 ** 31), 2 ** 31 - 1)}
+
+STATUS = {0: "QC_OK", 1: "QC_ERR_INVALID_ARG", 2: "QC_ERR_UNSUPPORTED", 3: "QC_ERR_OVERFLOW_RISK",
+          4: "QC_ERR_MISALIGNED", 5: "QC_ERR_WORKSPACE", 6: "QC_ERR_CUDA"}
+
+
+class QConvError(RuntimeError):
+    def __init__(self, fn: str, status: int, cuda_err: int = 0):
+        self.status = status
+        msg = f"{fn}: {STATUS.get(status, status)} ({_lib().qconv_status_string(status).decode()})"
+        if status == 6:
+            msg += f" cudaError={cuda_err}"
+        super().__init__(msg)
+
+
+class qconv_desc(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in
+                ("n", "h", "w", "c", "k", "r", "s", "stride_h", "stride_w", "pad_h", "pad_w",
+                 "dil_h", "dil_w", "x_t", "w_t", "y_t", "x_zero", "w_prepared", "y_zero",
+                 "clamp_lo", "clamp_hi")]
+
+
+_L = None
+
+
+def _lib():
+    global _L
+    if _L is None:
+        if not os.path.exists(_SO):
+            raise ImportError(f"libqconv.so not built at {_SO}; run __graft_entry__.build() "
+                              "(no CPU fallback exists)")
+        L = ctypes.CDLL(_SO)
+        vp, i32, i64, f32, sz = (ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_float,
+                                 ctypes.c_size_t)
+        dp = ctypes.POINTER(qconv_desc)
+        L.qconv_status_string.argtypes = [i32]
+        L.qconv_status_string.restype = ctypes.c_char_p
+        L.qconv_last_cuda_error.restype = i32
+        L.qconv_version.restype = i32
+        L.qconv_quantize_pack.argtypes = [vp, i32, i64, i32, i32, f32, i32, i32, vp, vp]
+        L.qconv_quantize_pack.restype = i32
+        L.qconv_requant_params.argtypes = [f32, vp, f32, i32, vp, vp]
+        L.qconv_requant_params.restype = i32
+        L.qconv_prepared_weight_bytes.argtypes = [dp]
+        L.qconv_prepared_weight_bytes.restype = sz
+        L.qconv_prepare_weights.argtypes = [dp, vp, vp, vp]
+        L.qconv_prepare_weights.restype = i32
+        L.qconv2d_workspace_size.argtypes = [dp]
+        L.qconv2d_workspace_size.restype = sz
+        L.qconv2d_forward.argtypes = [dp, vp, vp, vp, vp, vp, vp, vp, sz, vp]
+        L.qconv2d_forward.restype = i32
+        L.qconv_debug_im2col_tile.argtypes = [dp, vp, i64, i32, i32, i32, i32, vp, vp]
+        L.qconv_debug_im2col_tile.restype = i32
+        _L = L
+    return _L
+
+
+def lib_path() -> str:
+    return _SO
+
+
+def _check(fn: str, st: int):
+    if st != 0:
+        raise QConvError(fn, st, _lib().qconv_last_cuda_error())
+
+
+def _ptr(t) -> Optional[int]:
+    if t is None:
+        return None
+    return t.data_ptr()
+
+
+def _stream(stream) -> Optional[int]:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+
+
+# --------------------------------------------------------------------------- descriptors
+def make_desc(n, h, w, c, k, r, s, *, stride=1, pad=0, dil=1, x_t=QC_U8, w_t=QC_S8, y_t=QC_U8,
+              x_zero=0, w_prepared=0, y_zero=0, clamp_lo=None, clamp_hi=None,
+              relu=False) -> qconv_desc:
+    sh, sw = (stride, stride) if isinstance(stride, int) else stride
+    ph, pw = (pad, pad) if isinstance(pad, int) else pad
+    dh, dw = (dil, dil) if isinstance(dil, int) else dil
+    lo, hi = _RANGE[y_t] if y_t != QC_S32 else (0, 0)
+    if relu and y_t != QC_S32:
+        lo = max(lo, y_zero)
+    lo = lo if clamp_lo is None else clamp_lo
+    hi = hi if clamp_hi is None else clamp_hi
+    return qconv_desc(n, h, w, c, k, r, s, sh, sw, ph, pw, dh, dw, x_t, w_t, y_t, x_zero,
+                      w_prepared, y_zero, lo, hi)
+
+
+def out_hw(d: qconv_desc) -> Tuple[int, int]:
+    p = (d.h + 2 * d.pad_h - d.dil_h * (d.r - 1) - 1) // d.stride_h + 1
+    q = (d.w + 2 * d.pad_w - d.dil_w * (d.s - 1) - 1) // d.stride_w + 1
+    return p, q
+
+
+def output_nbytes_per_pixel(d: qconv_desc) -> int:
+    return d.k * _BITS[d.y_t] // 8
+
+
+# --------------------------------------------------------------------------- the C ABI
+def qconv_quantize_pack(x, scale: float, zero_point: int, yt: int, c_pad: Optional[int] = None,
+                        out=None, stream=None):
+    """x: CUDA tensor fp32/bf16 [..., C] -> uint8 [..., C_pad*bits/8] (include/qconv.h)."""
+    import torch
+    assert x.is_cuda and x.is_contiguous()
+    xt = QC_BF16 if x.dtype == torch.bfloat16 else QC_F32
+    assert x.dtype in (torch.float32, torch.bfloat16)
+    c = x.shape[-1]
+    c_pad = c if c_pad is None else c_pad
+    npix = x.numel() // c
+    nbytes = c_pad * _BITS[yt] // 8
+    if out is None:
+        out = torch.empty(tuple(x.shape[:-1]) + (nbytes,), dtype=torch.uint8, device=x.device)
+    _check("qconv_quantize_pack", _lib().qconv_quantize_pack(
+        _ptr(x), xt, npix, c, c_pad, float(scale), int(zero_point), int(yt), _ptr(out),
+        _stream(stream)))
+    return out
+
+
+def qconv_requant_params(in_scale: float, w_scale, out_scale: float):
+    """Host-only (reading R1) -> (multiplier int32[K], shift int32[K]) numpy arrays."""
+    ws = np.ascontiguousarray(np.asarray(w_scale, dtype=np.float32))
+    k = ws.shape[0]
+    m = np.zeros(k, dtype=np.int32)
+    n = np.zeros(k, dtype=np.int32)
+    _check("qconv_requant_params", _lib().qconv_requant_params(
+        float(in_scale), ws.ctypes.data, float(out_scale), k, m.ctypes.data, n.ctypes.data))
+    return m, n
+
+
+def qconv_prepared_weight_bytes(d: qconv_desc) -> int:
+    return int(_lib().qconv_prepared_weight_bytes(ctypes.byref(d)))
+
+
+def qconv_prepare_weights(d: qconv_desc, w, out=None, stream=None):
+    import torch
+    nb = qconv_prepared_weight_bytes(d)
+    if nb == 0:
+        raise QConvError("qconv_prepare_weights", 1)
+    if out is None:
+        out = torch.empty(nb, dtype=torch.uint8, device=w.device)
+    _check("qconv_prepare_weights", _lib().qconv_prepare_weights(
+        ctypes.byref(d), _ptr(w), _ptr(out), _stream(stream)))
+    return out
+
+
+def qconv2d_workspace_size(d: qconv_desc) -> int:
+    return int(_lib().qconv2d_workspace_size(ctypes.byref(d)))
+
+
+def qconv2d_forward(d: qconv_desc, x, w, bias=None, multiplier=None, shift=None, y=None,
+                    workspace=None, stream=None):
+    """y = requant(conv(x - x_zero, w) + bias) on the GPU (include/qconv.h)."""
+    import torch
+    if y is None:
+        p, q = out_hw(d)
+        if d.y_t == QC_S32:
+            y = torch.empty((d.n, p, q, d.k), dtype=torch.int32, device=x.device)
+        else:
+            y = torch.empty((d.n, p, q, output_nbytes_per_pixel(d)), dtype=torch.uint8,
+                            device=x.device)
+    ws_need = qconv2d_workspace_size(d)
+    if ws_need and workspace is None:
+        workspace = torch.empty(ws_need, dtype=torch.uint8, device=x.device)
+    ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
+    _check("qconv2d_forward", _lib().qconv2d_forward(
+        ctypes.byref(d), _ptr(x), _ptr(w), _ptr(bias), _ptr(multiplier), _ptr(shift), _ptr(y),
+        _ptr(workspace), ws_bytes, _stream(stream)))
+    return y
+
+
+def qconv_debug_im2col_tile(d: qconv_desc, x, m0: int, r: int, s: int, c_byte: int,
+                            box_bytes: int, stream=None):
+    import torch
+    out = torch.empty((128, box_bytes), dtype=torch.uint8, device=x.device)
+    _check("qconv_debug_im2col_tile", _lib().qconv_debug_im2col_tile(
+        ctypes.byref(d), _ptr(x), int(m0), int(r), int(s), int(c_byte), int(box_bytes),
+        _ptr(out), _stream(stream)))
+    return out
+
+
+# --------------------------------------------------------------------------- layer object
+@dataclass
+class QConv2d:
+    """A quantized conv layer resident on one GPU: prepared weights, bias and
+    requant parameters live in HBM; __call__ enqueues one qconv2d_forward."""
+    desc: qconv_desc
+    w_prep: object
+    bias: object
+    multiplier: object
+    shift: object
+    workspace: object = None
+
+    @classmethod
+    def create(cls, desc: qconv_desc, w_bytes, bias, multiplier, shift, device="cuda",
+               stream=None):
+        import torch
+        w_dev = torch.as_tensor(np.ascontiguousarray(w_bytes)).to(device)
+        w_prep = qconv_prepare_weights(desc, w_dev, stream=stream)
+        d = qconv_desc.from_buffer_copy(desc)
+        d.w_prepared = 1
+        b = None if bias is None else torch.as_tensor(np.asarray(bias, np.int32)).to(device)
+        m = None if multiplier is None else torch.as_tensor(np.asarray(multiplier, np.int32)).to(device)
+        s = None if shift is None else torch.as_tensor(np.asarray(shift, np.int32)).to(device)
+        ws = qconv2d_workspace_size(d)
+        wsb = torch.empty(ws, dtype=torch.uint8, device=device) if ws else None
+        return cls(d, w_prep, b, m, s, wsb)
+
+    def __call__(self, x, y=None, stream=None):
+        return qconv2d_forward(self.desc, x, self.w_prep, self.bias, self.multiplier, self.shift,
+                               y=y, workspace=self.workspace, stream=stream)
+
+
+__all__ = ["qconv_quantize_pack", "qconv_requant_params", "qconv_prepare_weights",
+           "qconv_prepared_weight_bytes", "qconv2d_workspace_size", "qconv2d_forward",
+           "qconv_debug_im2col_tile", "make_desc", "qconv_desc", "QConv2d", "QConvError",
+           "QC_U4", "QC_S4", "QC_U8", "QC_S8", "QC_S32", "out_hw", "lib_path"]
+
+_lib()   # fail loudly at import if the CUDA library is missing

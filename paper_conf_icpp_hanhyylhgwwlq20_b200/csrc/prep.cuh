@@ -1,0 +1,153 @@
+// prep.cuh -- memory-bound kernels around the convolution:
+//   quantize_pack_kernel : fp32/bf16 NHWC -> packed int8/int4 NHWC (Z4)
+//   widen_w4_kernel      : packed int4 KRSC weights -> int8 KRSC (once per layer)
+//   zx_table_kernel      : 2-D prefix sums of sum_c w[k,r,s,c] for x_zero != 0 borders (Z2)
+#pragma once
+#include <cstdint>
+#include <cuda_bf16.h>
+
+namespace qc {
+
+struct QuantParams {
+    const void *x;
+    void *y;
+    int64_t npix;
+    int32_t c, c_pad;
+    float inv_s;        // fl32(1/scale), computed on the host in fp32
+    float flo, fhi;     // qmin - z - 1, qmax - z + 1 (pre-clamp keeps the int conversion exact)
+    int32_t z, qmin, qmax;
+    int32_t bf16, bits;
+    int32_t fast;       // c == c_pad, c % 16 == 0, 16-byte aligned rows
+};
+
+__device__ __forceinline__ int32_t quantize_one(float x, const QuantParams &p) {
+    float t = __fmul_rn(x, p.inv_s);                 // one IEEE fp32 multiply, RNE
+    if (isnan(t)) return p.z;
+    t = fminf(fmaxf(t, p.flo), p.fhi);
+    const int32_t q = __float2int_rn(t) + p.z;       // round half to even
+    return min(p.qmax, max(p.qmin, q));
+}
+
+__device__ __forceinline__ float load_x(const QuantParams &p, int64_t i) {
+    if (p.bf16) {
+        const uint16_t b = static_cast<const uint16_t *>(p.x)[i];
+        return __uint_as_float(static_cast<uint32_t>(b) << 16);
+    }
+    return static_cast<const float *>(p.x)[i];
+}
+
+// One thread = 16 consecutive output elements (16 B of int8 or 8 B of int4).
+__global__ void __launch_bounds__(256) quantize_pack_kernel(const __grid_constant__ QuantParams p) {
+    const int64_t total = p.npix * p.c_pad;
+    const int64_t ngroups = (total + 15) / 16;
+    for (int64_t g = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; g < ngroups;
+         g += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t e0 = g * 16;
+        int32_t q[16];
+        if (p.fast && e0 + 16 <= total) {
+            if (p.bf16) {
+                const uint4 *src = reinterpret_cast<const uint4 *>(static_cast<const uint16_t *>(p.x) + e0);
+                const uint4 a = __ldg(src), b = __ldg(src + 1);
+                const uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    q[2 * j] = quantize_one(__uint_as_float(w[j] << 16), p);
+                    q[2 * j + 1] = quantize_one(__uint_as_float(w[j] & 0xFFFF0000u), p);
+                }
+            } else {
+                const float4 *src = reinterpret_cast<const float4 *>(static_cast<const float *>(p.x) + e0);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const float4 v = __ldg(src + j);
+                    q[4 * j] = quantize_one(v.x, p);
+                    q[4 * j + 1] = quantize_one(v.y, p);
+                    q[4 * j + 2] = quantize_one(v.z, p);
+                    q[4 * j + 3] = quantize_one(v.w, p);
+                }
+            }
+        } else {
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+                const int64_t e = e0 + j;
+                if (e < total) {
+                    const int64_t pix = e / p.c_pad;
+                    const int32_t ch = static_cast<int32_t>(e - pix * p.c_pad);
+                    q[j] = ch < p.c ? quantize_one(load_x(p, pix * p.c + ch), p) : p.z;
+                } else {
+                    q[j] = 0;
+                }
+            }
+        }
+        if (p.bits == 8) {
+            uint32_t w[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                w[j] = (q[4 * j] & 0xFF) | ((q[4 * j + 1] & 0xFF) << 8) | ((q[4 * j + 2] & 0xFF) << 16) |
+                       (static_cast<uint32_t>(q[4 * j + 3] & 0xFF) << 24);
+            uint8_t *dst = static_cast<uint8_t *>(p.y) + e0;
+            if (e0 + 16 <= total && (reinterpret_cast<uintptr_t>(dst) & 15u) == 0) {
+                *reinterpret_cast<uint4 *>(dst) = make_uint4(w[0], w[1], w[2], w[3]);
+            } else {
+                for (int j = 0; j < 16 && e0 + j < total; ++j) dst[j] = static_cast<uint8_t>(q[j] & 0xFF);
+            }
+        } else {
+            uint32_t w[2];
+#pragma unroll
+            for (int j = 0; j < 2; ++j) {
+                uint32_t acc = 0;
+#pragma unroll
+                for (int i = 0; i < 8; ++i) acc |= static_cast<uint32_t>(q[8 * j + i] & 0xF) << (4 * i);
+                w[j] = acc;
+            }
+            uint8_t *dst = static_cast<uint8_t *>(p.y) + e0 / 2;
+            if (e0 + 16 <= total && (reinterpret_cast<uintptr_t>(dst) & 7u) == 0) {
+                *reinterpret_cast<uint2 *>(dst) = make_uint2(w[0], w[1]);
+            } else {
+                for (int j = 0; 2 * j < 16 && e0 + 2 * j < total; ++j)
+                    dst[j] = static_cast<uint8_t>((q[2 * j] & 0xF) | ((q[2 * j + 1] & 0xF) << 4));
+            }
+        }
+    }
+}
+
+// packed int4 -> int8 (sign- or zero-extended); n_bytes_in packed bytes.
+__global__ void __launch_bounds__(256) widen_w4_kernel(const uint8_t *__restrict__ w4,
+                                                       int8_t *__restrict__ w8, int64_t n_bytes_in,
+                                                       int32_t is_signed) {
+    for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n_bytes_in;
+         i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const uint8_t b = w4[i];
+        int lo = b & 0xF, hi = b >> 4;
+        if (is_signed) {
+            lo = lo >= 8 ? lo - 16 : lo;
+            hi = hi >= 8 ? hi - 16 : hi;
+        }
+        w8[2 * i] = static_cast<int8_t>(lo);
+        w8[2 * i + 1] = static_cast<int8_t>(hi);
+    }
+}
+
+// table[k][i][j] = sum_{r<i, s<j} sum_c w8[k,r,s,c]  (i in [0,R], j in [0,S]).
+// For an output pixel whose in-bounds taps are r in [r0,r1), s in [s0,s1) the
+// padded taps' contribution to subtract is x_zero * (T[r1][s1]-T[r0][s1]-T[r1][s0]+T[r0][s0]).
+__global__ void zx_table_kernel(const int8_t *__restrict__ w8, int32_t *__restrict__ table, int K,
+                                int R, int S, int C, int is_unsigned) {
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= K) return;
+    int32_t *t = table + static_cast<int64_t>(k) * (R + 1) * (S + 1);
+    for (int j = 0; j <= S; ++j) t[j] = 0;
+    for (int i = 1; i <= R; ++i) {
+        t[i * (S + 1)] = 0;
+        int32_t rowsum = 0;
+        for (int j = 1; j <= S; ++j) {
+            const int8_t *src = w8 + ((static_cast<int64_t>(k) * R + (i - 1)) * S + (j - 1)) * C;
+            int32_t s = 0;
+            for (int c = 0; c < C; ++c) s += is_unsigned ? static_cast<int32_t>(static_cast<uint8_t>(src[c]))
+                                                         : static_cast<int32_t>(src[c]);
+            rowsum += s;
+            t[i * (S + 1) + j] = t[(i - 1) * (S + 1) + j] + rowsum;
+        }
+    }
+}
+
+}  // namespace qc

@@ -1,0 +1,569 @@
+// qconv.cu -- host side of libqconv.so: the C ABI declared in include/qconv.h.
+//
+// Validation, the overflow bound, the per-shape launch plan (tile sizes,
+// pipeline depth, shared-memory carve-up), TMA descriptor encoding (im2col
+// for activations, tiled for weights) and kernel launches.  All device work
+// is in conv_fwd.cuh / prep.cuh.  Nothing here allocates device memory.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+
+#include "qconv.h"
+#include "conv_fwd.cuh"
+#include "prep.cuh"
+
+namespace {
+
+thread_local int g_last_cuda_error = 0;
+
+qc_status cuda_fail(cudaError_t e) {
+    g_last_cuda_error = static_cast<int>(e);
+    return QC_ERR_CUDA;
+}
+
+bool is_int_input(qc_dtype t) { return t == QC_U4 || t == QC_S4 || t == QC_U8 || t == QC_S8; }
+bool is_valid_dtype(qc_dtype t) { return is_int_input(t) || t == QC_S32; }
+int dtype_bits(qc_dtype t) { return (t == QC_U4 || t == QC_S4) ? 4 : (t == QC_S32 ? 32 : 8); }
+bool dtype_signed(qc_dtype t) { return t == QC_S4 || t == QC_S8 || t == QC_S32; }
+int64_t dtype_min(qc_dtype t) {
+    switch (t) {
+        case QC_U4: return 0;
+        case QC_S4: return -8;
+        case QC_U8: return 0;
+        case QC_S8: return -128;
+        default: return INT32_MIN;
+    }
+}
+int64_t dtype_max(qc_dtype t) {
+    switch (t) {
+        case QC_U4: return 15;
+        case QC_S4: return 7;
+        case QC_U8: return 255;
+        case QC_S8: return 127;
+        default: return INT32_MAX;
+    }
+}
+bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+// ------------------------------------------------------------------ driver entry points
+typedef CUresult (*PFN_encodeIm2col)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                     const cuuint64_t *, const cuuint64_t *, const int *,
+                                     const int *, cuuint32_t, cuuint32_t, const cuuint32_t *,
+                                     CUtensorMapInterleave, CUtensorMapSwizzle,
+                                     CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                    const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                                    const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                    CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+struct Driver {
+    PFN_encodeIm2col im2col = nullptr;
+    PFN_encodeTiled tiled = nullptr;
+    int driver_version = 0;
+    cudaError_t err = cudaSuccess;
+};
+
+const Driver &driver() {
+    static Driver d;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void *f1 = nullptr, *f2 = nullptr;
+        cudaDriverEntryPointQueryResult q1, q2;
+        cudaError_t e1 = cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &f1, cudaEnableDefault, &q1);
+        cudaError_t e2 = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f2, cudaEnableDefault, &q2);
+        if (e1 != cudaSuccess || e2 != cudaSuccess || q1 != cudaDriverEntryPointSuccess ||
+            q2 != cudaDriverEntryPointSuccess) {
+            d.err = e1 != cudaSuccess ? e1 : (e2 != cudaSuccess ? e2 : cudaErrorSymbolNotFound);
+            return;
+        }
+        d.im2col = reinterpret_cast<PFN_encodeIm2col>(f1);
+        d.tiled = reinterpret_cast<PFN_encodeTiled>(f2);
+        cudaDriverGetVersion(&d.driver_version);
+    });
+    return d;
+}
+
+// Driver releases up to 13.1 mis-handle a descriptor flag for tensors under
+// 128 KiB; clearing bit 21 of the second descriptor word is the documented
+// workaround used by NVIDIA's own TMA helpers.
+void small_tensor_fixup(CUtensorMap *m, uint64_t tensor_bytes) {
+    if (driver().driver_version <= 13010 && tensor_bytes < 131072)
+        reinterpret_cast<uint64_t *>(m)[1] &= ~(1ull << 21);
+}
+
+int num_sms() {
+    static int cache[64] = {0};
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (cache[dev] == 0) {
+        int n = 0;
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        cache[dev] = n > 0 ? n : 148;
+    }
+    return cache[dev];
+}
+
+// ------------------------------------------------------------------ descriptor validation
+struct Geometry {
+    int P, Q;
+    int64_t M;
+    int bits;
+    int c_bytes;        // packed bytes per input pixel
+    int64_t x_bytes, w_bytes, w8_bytes, y_bytes;
+};
+
+qc_status validate_desc(const qconv_desc *d, Geometry *g) {
+    if (!d) return QC_ERR_INVALID_ARG;
+    if (d->n < 1 || d->h < 1 || d->w < 1 || d->c < 1 || d->k < 1 || d->r < 1 || d->s < 1)
+        return QC_ERR_INVALID_ARG;
+    if (d->stride_h < 1 || d->stride_w < 1 || d->dil_h < 1 || d->dil_w < 1 || d->pad_h < 0 ||
+        d->pad_w < 0)
+        return QC_ERR_INVALID_ARG;
+    if (!is_int_input(d->x_t) || !is_int_input(d->w_t) || !is_valid_dtype(d->y_t))
+        return QC_ERR_INVALID_ARG;
+    const int P = (d->h + 2 * d->pad_h - d->dil_h * (d->r - 1) - 1) / d->stride_h + 1;
+    const int Q = (d->w + 2 * d->pad_w - d->dil_w * (d->s - 1) - 1) / d->stride_w + 1;
+    if (d->h + 2 * d->pad_h - d->dil_h * (d->r - 1) - 1 < 0 ||
+        d->w + 2 * d->pad_w - d->dil_w * (d->s - 1) - 1 < 0 || P < 1 || Q < 1)
+        return QC_ERR_INVALID_ARG;
+    if (d->x_zero < dtype_min(d->x_t) || d->x_zero > dtype_max(d->x_t)) return QC_ERR_INVALID_ARG;
+    if (d->y_t != QC_S32) {
+        if (d->y_zero < dtype_min(d->y_t) || d->y_zero > dtype_max(d->y_t)) return QC_ERR_INVALID_ARG;
+        if (d->clamp_lo > d->clamp_hi || d->clamp_lo < dtype_min(d->y_t) ||
+            d->clamp_hi > dtype_max(d->y_t))
+            return QC_ERR_INVALID_ARG;
+    }
+    const int bits = dtype_bits(d->x_t);
+    if (bits == 4 && (d->c % 2)) return QC_ERR_INVALID_ARG;
+    const int64_t M = static_cast<int64_t>(d->n) * P * Q;
+    g->P = P;
+    g->Q = Q;
+    g->M = M;
+    g->bits = bits;
+    g->c_bytes = d->c * bits / 8;
+    g->x_bytes = static_cast<int64_t>(d->n) * d->h * d->w * g->c_bytes;
+    g->w8_bytes = static_cast<int64_t>(d->k) * d->r * d->s * d->c;
+    g->w_bytes = g->w8_bytes * dtype_bits(d->w_t) / 8;
+    const int yb = dtype_bits(d->y_t);
+    if (yb == 4 && (d->k % 2)) return QC_ERR_UNSUPPORTED;
+    g->y_bytes = M * d->k * yb / 8;
+    return QC_OK;
+}
+
+// Support + overflow checks for the GPU path (after validate_desc).
+qc_status check_supported(const qconv_desc *d, const Geometry &g) {
+    if (dtype_bits(d->x_t) != dtype_bits(d->w_t)) return QC_ERR_UNSUPPORTED;   // mixed widths: NEXT
+    if (d->c % 32) return QC_ERR_UNSUPPORTED;          // MMA K granularity / 16-byte TMA strides
+    if (d->stride_h > 8 || d->stride_w > 8) return QC_ERR_UNSUPPORTED;   // TMA traversal stride
+    const int lw = -d->pad_w, lh = -d->pad_h;
+    const int uw = d->pad_w - d->dil_w * (d->s - 1), uh = d->pad_h - d->dil_h * (d->r - 1);
+    if (lw < -128 || lh < -128 || uw < -128 || uh < -128 || uw > 127 || uh > 127)
+        return QC_ERR_UNSUPPORTED;                     // rank-4 im2col corner range
+    if (d->dil_w * (d->s - 1) > 255 || d->dil_h * (d->r - 1) > 255) return QC_ERR_UNSUPPORTED;
+    if (g.M > INT32_MAX - 256 || d->n > 65535) return QC_ERR_UNSUPPORTED;
+    if (static_cast<int64_t>(d->r) * d->s * d->c > INT32_MAX / 2) return QC_ERR_UNSUPPORTED;
+    // int32 accumulation bound ("overflow well addressed"): both the raw MMA sum and the
+    // zero-point-centred sum must stay inside int32 for any codes of these dtypes.
+    const int64_t T = static_cast<int64_t>(d->r) * d->s * d->c;
+    const int64_t wmax = std::max(-dtype_min(d->w_t), dtype_max(d->w_t));
+    const int64_t xraw = std::max(-dtype_min(d->x_t), dtype_max(d->x_t));
+    const int64_t xctr = std::max(d->x_zero - dtype_min(d->x_t), dtype_max(d->x_t) - d->x_zero);
+    const double lim = 2147483647.0;
+    if (static_cast<double>(T) * xraw * wmax > lim || static_cast<double>(T) * xctr * wmax > lim)
+        return QC_ERR_OVERFLOW_RISK;
+    return QC_OK;
+}
+
+// ------------------------------------------------------------------ launch plan
+struct Plan {
+    int BK, bkp, chunks, BN, n_tiles_n, num_tiles, num_kb, stages, grid, threads;
+    uint32_t tmem_cols, smem_bytes;
+    qc::ConvParams cp;
+};
+
+int choose_bk(int c) { return (c % 128 == 0) ? 128 : (c % 64 == 0 ? 64 : 32); }
+uint32_t pow2_cols(int n) {
+    uint32_t c = 32;
+    while (c < static_cast<uint32_t>(n)) c <<= 1;
+    return c;
+}
+
+qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
+    const bool is4 = g.bits == 4;
+    pl->BK = choose_bk(d->c);
+    pl->bkp = is4 ? pl->BK / 2 : pl->BK;
+    pl->chunks = d->c / pl->BK;
+    pl->num_kb = d->r * d->s * pl->chunks;
+    const int m_tiles = static_cast<int>((g.M + qc::kBM - 1) / qc::kBM);
+    const int sms = num_sms();
+    int BN = std::min(qc::kMaxBN, ((d->k + 15) / 16) * 16);
+    // smaller N tiles when the grid would not fill the GPU (paper P:L321: at small batch the
+    // tiling decides how well the machine is filled)
+    while (BN > 64 && static_cast<int64_t>(m_tiles) * ((d->k + BN - 1) / BN) < sms) {
+        BN = std::max(64, ((BN / 2 + 15) / 16) * 16);
+    }
+    pl->BN = BN;
+    pl->n_tiles_n = (d->k + BN - 1) / BN;
+    pl->num_tiles = m_tiles * pl->n_tiles_n;
+    pl->tmem_cols = pow2_cols(2 * BN);
+    const uint32_t a_bytes = static_cast<uint32_t>(qc::kBM * pl->BK);
+    const uint32_t b_bytes = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * pl->BK, 1024));
+    const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(qc::kBM * pl->bkp) : 0u;
+    const uint32_t per_stage = a_bytes + b_bytes + stg_bytes;
+    const uint32_t fixed = static_cast<uint32_t>(BN) * 16u + 1024u;     // params + barriers
+    const uint32_t budget = 227u * 1024u - 1024u - fixed;
+    int stages = static_cast<int>(budget / per_stage);
+    stages = std::min(stages, 8);
+    if (stages < 2) return QC_ERR_UNSUPPORTED;
+    pl->stages = stages;
+    qc::ConvParams &p = pl->cp;
+    std::memset(&p, 0, sizeof(p));
+    p.off_a = 0;
+    p.off_b = p.off_a + a_bytes * stages;
+    p.off_stg = p.off_b + b_bytes * stages;
+    p.off_par = static_cast<uint32_t>(align_up(p.off_stg + stg_bytes * stages, 16));
+    p.off_bar = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(BN) * 16u, 8));
+    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 4) * 8 + 16);
+    pl->smem_bytes = p.off_bar + bar_bytes + 1024u;       // + alignment slack for the 1024-B base
+    pl->grid = std::min(pl->num_tiles, sms);
+    pl->threads = is4 ? 384 : 256;
+    p.a_stage_bytes = a_bytes;
+    p.b_stage_bytes = b_bytes;
+    p.stg_stage_bytes = stg_bytes;
+    p.M = static_cast<int32_t>(g.M);
+    p.P = g.P;
+    p.Q = g.Q;
+    p.PQ = g.P * g.Q;
+    p.K = d->k;
+    p.BN = BN;
+    p.n_tiles_n = pl->n_tiles_n;
+    p.num_tiles = pl->num_tiles;
+    p.num_kb = pl->num_kb;
+    p.chunks = pl->chunks;
+    p.S = d->s;
+    p.R = d->r;
+    p.stride_h = d->stride_h;
+    p.stride_w = d->stride_w;
+    p.pad_h = d->pad_h;
+    p.pad_w = d->pad_w;
+    p.dil_h = d->dil_h;
+    p.dil_w = d->dil_w;
+    p.H = d->h;
+    p.W = d->w;
+    p.C8 = d->c;
+    p.BK = pl->BK;
+    p.bkp = pl->bkp;
+    p.stages = stages;
+    p.sw_layout = pl->BK == 128 ? 2 : (pl->BK == 64 ? 4 : 6);
+    p.sw_mask = pl->BK == 128 ? 7 : (pl->BK == 64 ? 3 : 1);
+    p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), dtype_signed(d->x_t), dtype_signed(d->w_t));
+    p.tmem_cols = pl->tmem_cols;
+    p.y_zero = d->y_t == QC_S32 ? 0 : d->y_zero;
+    p.clamp_lo = d->y_t == QC_S32 ? INT32_MIN : d->clamp_lo;
+    p.clamp_hi = d->y_t == QC_S32 ? INT32_MAX : d->clamp_hi;
+    p.x_zero = d->x_zero;
+    p.y_row_bytes = static_cast<int64_t>(d->k) * dtype_bits(d->y_t) / 8;
+    return QC_OK;
+}
+
+CUtensorMapSwizzle swizzle_for(int bk) {
+    return bk == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                     : (bk == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B);
+}
+
+qc_status encode_x_map(const qconv_desc *d, const Geometry &g, const void *x, int box_bytes,
+                       CUtensorMapSwizzle sw, CUtensorMap *map) {
+    const Driver &drv = driver();
+    if (!drv.im2col) return cuda_fail(drv.err);
+    const cuuint64_t cb = static_cast<cuuint64_t>(g.c_bytes);
+    cuuint64_t dims[4] = {cb, static_cast<cuuint64_t>(d->w), static_cast<cuuint64_t>(d->h),
+                          static_cast<cuuint64_t>(d->n)};
+    cuuint64_t strides[3] = {cb, cb * d->w, cb * d->w * d->h};
+    int lower[2] = {-d->pad_w, -d->pad_h};
+    int upper[2] = {d->pad_w - d->dil_w * (d->s - 1), d->pad_h - d->dil_h * (d->r - 1)};
+    cuuint32_t estr[4] = {1, static_cast<cuuint32_t>(d->stride_w), static_cast<cuuint32_t>(d->stride_h), 1};
+    CUresult r = drv.im2col(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, const_cast<void *>(x), dims,
+                            strides, lower, upper, static_cast<cuuint32_t>(box_bytes),
+                            static_cast<cuuint32_t>(qc::kBM), estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+    small_tensor_fixup(map, static_cast<uint64_t>(g.x_bytes));
+    return QC_OK;
+}
+
+qc_status encode_w_map(const qconv_desc *d, const Geometry &g, const void *w8, int bk, int bn,
+                       CUtensorMap *map) {
+    const Driver &drv = driver();
+    if (!drv.tiled) return cuda_fail(drv.err);
+    const cuuint64_t kg = static_cast<cuuint64_t>(d->r) * d->s * d->c;
+    cuuint64_t dims[2] = {kg, static_cast<cuuint64_t>(d->k)};
+    cuuint64_t strides[1] = {kg};
+    cuuint32_t box[2] = {static_cast<cuuint32_t>(bk), static_cast<cuuint32_t>(bn)};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = drv.tiled(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<void *>(w8), dims,
+                           strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_for(bk),
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+    small_tensor_fixup(map, static_cast<uint64_t>(g.w8_bytes));
+    return QC_OK;
+}
+
+template <bool IS4, int OUT>
+qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
+                      cudaStream_t stream) {
+    auto kern = qc::qconv_fwd_kernel<IS4, OUT>;
+    static int configured_smem = 0;   // per instantiation; max over calls is safe to keep
+    if (configured_smem < static_cast<int>(pl.smem_bytes)) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             227 * 1024);
+        if (e != cudaSuccess) return cuda_fail(e);
+        configured_smem = 227 * 1024;
+    }
+    cudaLaunchConfig_t cfg;
+    std::memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
+    cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
+    cfg.dynamicSmemBytes = pl.smem_bytes;
+    cfg.stream = stream;
+    cfg.attrs = nullptr;
+    cfg.numAttrs = 0;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, pl.cp);
+    if (e != cudaSuccess) return cuda_fail(e);
+    return QC_OK;
+}
+
+}  // namespace
+
+// ====================================================================== C ABI
+extern "C" {
+
+const char *qconv_status_string(qc_status s) {
+    switch (s) {
+        case QC_OK: return "ok";
+        case QC_ERR_INVALID_ARG: return "invalid argument";
+        case QC_ERR_UNSUPPORTED: return "unsupported configuration";
+        case QC_ERR_OVERFLOW_RISK: return "int32 accumulator overflow risk";
+        case QC_ERR_MISALIGNED: return "device pointer not 16-byte aligned";
+        case QC_ERR_WORKSPACE: return "workspace missing or too small";
+        case QC_ERR_CUDA: return "CUDA error";
+    }
+    return "unknown status";
+}
+
+int qconv_last_cuda_error(void) { return g_last_cuda_error; }
+int qconv_version(void) { return 100; }
+
+qc_status qconv_requant_params(float in_scale, const float *w_scale, float out_scale, int32_t k,
+                               int32_t *multiplier, int32_t *shift) {
+    if (!w_scale || !multiplier || !shift || k < 1) return QC_ERR_INVALID_ARG;
+    if (!(in_scale > 0.0f) || !(out_scale > 0.0f) || !std::isfinite(in_scale) ||
+        !std::isfinite(out_scale))
+        return QC_ERR_INVALID_ARG;
+    for (int32_t i = 0; i < k; ++i) {
+        const float ws = w_scale[i];
+        if (!(ws >= 0.0f) || !std::isfinite(ws)) return QC_ERR_INVALID_ARG;
+        // exact product of two binary32 values in binary64, then one RNE division
+        const double M = (static_cast<double>(in_scale) * static_cast<double>(ws)) /
+                         static_cast<double>(out_scale);
+        if (M == 0.0) {
+            multiplier[i] = 0;
+            shift[i] = 31;
+            continue;
+        }
+        int e = 0;
+        const double f = std::frexp(M, &e);                   // M = f * 2^e, f in [0.5, 1)
+        const double scaled = std::ldexp(f, 31);              // exact
+        int64_t m = static_cast<int64_t>(scaled);             // floor (scaled > 0)
+        if (scaled - static_cast<double>(m) >= 0.5) m += 1;   // round half up
+        if (m == (int64_t(1) << 31)) {
+            m = int64_t(1) << 30;
+            e += 1;
+        }
+        const int n = 31 - e;
+        if (n < 1 || n > 62) return QC_ERR_INVALID_ARG;
+        multiplier[i] = static_cast<int32_t>(m);
+        shift[i] = n;
+    }
+    return QC_OK;
+}
+
+qc_status qconv_quantize_pack(const void *x, qc_ftype xt, int64_t npix, int32_t c, int32_t c_pad,
+                              float scale, int32_t zero_point, qc_dtype yt, void *y, void *stream) {
+    if (!x || !y || npix < 0 || c < 1 || c_pad < c) return QC_ERR_INVALID_ARG;
+    if (xt != QC_F32 && xt != QC_BF16) return QC_ERR_INVALID_ARG;
+    if (!is_int_input(yt)) return QC_ERR_INVALID_ARG;
+    if (!(scale > 0.0f) || !std::isfinite(scale)) return QC_ERR_INVALID_ARG;
+    if (zero_point < dtype_min(yt) || zero_point > dtype_max(yt)) return QC_ERR_INVALID_ARG;
+    const int bits = dtype_bits(yt);
+    if (bits == 4 && (c_pad % 2)) return QC_ERR_INVALID_ARG;
+    if (!aligned16(x) || !aligned16(y)) return QC_ERR_MISALIGNED;
+    if (npix == 0) return QC_OK;
+    qc::QuantParams p;
+    p.x = x;
+    p.y = y;
+    p.npix = npix;
+    p.c = c;
+    p.c_pad = c_pad;
+    p.inv_s = 1.0f / scale;
+    p.z = zero_point;
+    p.qmin = static_cast<int32_t>(dtype_min(yt));
+    p.qmax = static_cast<int32_t>(dtype_max(yt));
+    p.flo = static_cast<float>(p.qmin - p.z - 1);
+    p.fhi = static_cast<float>(p.qmax - p.z + 1);
+    p.bf16 = xt == QC_BF16;
+    p.bits = bits;
+    p.fast = (c == c_pad) && (c % 16 == 0);
+    const int64_t groups = (npix * c_pad + 15) / 16;
+    const int64_t blocks_needed = (groups + 255) / 256;
+    const int grid = static_cast<int>(std::min<int64_t>(blocks_needed, static_cast<int64_t>(num_sms()) * 8));
+    qc::quantize_pack_kernel<<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(p);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e);
+    return QC_OK;
+}
+
+size_t qconv_prepared_weight_bytes(const qconv_desc *d) {
+    Geometry g;
+    if (validate_desc(d, &g) != QC_OK) return 0;
+    return static_cast<size_t>(g.w8_bytes);
+}
+
+static qc_status prepare_weights_impl(const qconv_desc *d, const Geometry &g, const void *w,
+                                      void *w_prep, cudaStream_t st) {
+    if (dtype_bits(d->w_t) == 8) {
+        cudaError_t e = cudaMemcpyAsync(w_prep, w, static_cast<size_t>(g.w8_bytes),
+                                        cudaMemcpyDeviceToDevice, st);
+        if (e != cudaSuccess) return cuda_fail(e);
+        return QC_OK;
+    }
+    const int64_t nin = g.w8_bytes / 2;
+    const int grid = static_cast<int>(std::min<int64_t>((nin + 255) / 256, 4096));
+    qc::widen_w4_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(w),
+                                              static_cast<int8_t *>(w_prep), nin,
+                                              d->w_t == QC_S4 ? 1 : 0);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e);
+    return QC_OK;
+}
+
+qc_status qconv_prepare_weights(const qconv_desc *d, const void *w, void *w_prep, void *stream) {
+    Geometry g;
+    qc_status s = validate_desc(d, &g);
+    if (s != QC_OK) return s;
+    if (!w || !w_prep) return QC_ERR_INVALID_ARG;
+    if (!aligned16(w) || !aligned16(w_prep)) return QC_ERR_MISALIGNED;
+    return prepare_weights_impl(d, g, w, w_prep, static_cast<cudaStream_t>(stream));
+}
+
+static size_t ws_weights_bytes(const qconv_desc *d, const Geometry &g) {
+    return (dtype_bits(d->w_t) == 4 && !d->w_prepared) ? align_up(static_cast<size_t>(g.w8_bytes), 256) : 0;
+}
+static size_t ws_zx_bytes(const qconv_desc *d) {
+    return d->x_zero != 0 ? align_up(static_cast<size_t>(d->k) * (d->r + 1) * (d->s + 1) * 4, 256) : 0;
+}
+
+size_t qconv2d_workspace_size(const qconv_desc *d) {
+    Geometry g;
+    if (validate_desc(d, &g) != QC_OK) return 0;
+    return ws_weights_bytes(d, g) + ws_zx_bytes(d);
+}
+
+qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, const int32_t *bias,
+                          const int32_t *multiplier, const int32_t *shift, void *y, void *workspace,
+                          size_t ws_bytes, void *stream) {
+    Geometry g;
+    qc_status s = validate_desc(d, &g);
+    if (s != QC_OK) return s;
+    if (!x || !w || !y) return QC_ERR_INVALID_ARG;
+    if (d->y_t != QC_S32 && (!multiplier || !shift)) return QC_ERR_INVALID_ARG;
+    s = check_supported(d, g);
+    if (s != QC_OK) return s;
+    if (!aligned16(x) || !aligned16(w) || !aligned16(y) || (bias && !aligned16(bias)) ||
+        (multiplier && !aligned16(multiplier)) || (shift && !aligned16(shift)) ||
+        (workspace && !aligned16(workspace)))
+        return QC_ERR_MISALIGNED;
+    const size_t need_w = ws_weights_bytes(d, g), need_z = ws_zx_bytes(d);
+    if (need_w + need_z > 0 && (!workspace || ws_bytes < need_w + need_z)) return QC_ERR_WORKSPACE;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+
+    Plan pl;
+    s = make_plan(d, g, &pl);
+    if (s != QC_OK) return s;
+
+    const void *w8 = w;
+    if (need_w) {
+        s = prepare_weights_impl(d, g, w, workspace, st);
+        if (s != QC_OK) return s;
+        w8 = workspace;
+    }
+    qc::ConvParams &p = pl.cp;
+    if (need_z) {
+        int32_t *table = reinterpret_cast<int32_t *>(static_cast<uint8_t *>(workspace) + need_w);
+        qc::zx_table_kernel<<<(d->k + 127) / 128, 128, 0, st>>>(
+            static_cast<const int8_t *>(w8), table, d->k, d->r, d->s, d->c, dtype_signed(d->w_t) ? 0 : 1);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_fail(e);
+        p.zx_table = table;
+    }
+    p.bias = bias;
+    p.mult = multiplier;
+    p.shift = shift;
+    p.y = y;
+
+    alignas(64) CUtensorMap xm, wm;
+    s = encode_x_map(d, g, x, pl.bkp, g.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(pl.BK), &xm);
+    if (s != QC_OK) return s;
+    s = encode_w_map(d, g, w8, pl.BK, pl.BN, &wm);
+    if (s != QC_OK) return s;
+
+    const bool is4 = g.bits == 4;
+    switch (d->y_t) {
+        case QC_S32: return is4 ? launch_conv<true, qc::OUT_S32>(pl, xm, wm, st) : launch_conv<false, qc::OUT_S32>(pl, xm, wm, st);
+        case QC_U8: return is4 ? launch_conv<true, qc::OUT_U8>(pl, xm, wm, st) : launch_conv<false, qc::OUT_U8>(pl, xm, wm, st);
+        case QC_S8: return is4 ? launch_conv<true, qc::OUT_S8>(pl, xm, wm, st) : launch_conv<false, qc::OUT_S8>(pl, xm, wm, st);
+        case QC_U4: return is4 ? launch_conv<true, qc::OUT_U4>(pl, xm, wm, st) : launch_conv<false, qc::OUT_U4>(pl, xm, wm, st);
+        case QC_S4: return is4 ? launch_conv<true, qc::OUT_S4>(pl, xm, wm, st) : launch_conv<false, qc::OUT_S4>(pl, xm, wm, st);
+    }
+    return QC_ERR_INVALID_ARG;
+}
+
+qc_status qconv_debug_im2col_tile(const qconv_desc *d, const void *x, int64_t m0, int32_t r,
+                                  int32_t s_, int32_t c_byte, int32_t box_bytes, void *out,
+                                  void *stream) {
+    Geometry g;
+    qc_status s = validate_desc(d, &g);
+    if (s != QC_OK) return s;
+    if (!x || !out || m0 < 0 || m0 >= g.M || r < 0 || r >= d->r || s_ < 0 || s_ >= d->s ||
+        box_bytes < 16 || box_bytes > 256 || box_bytes % 16 || c_byte < 0 ||
+        c_byte + box_bytes > g.c_bytes)
+        return QC_ERR_INVALID_ARG;
+    if (g.c_bytes % 16) return QC_ERR_UNSUPPORTED;
+    alignas(64) CUtensorMap xm;
+    s = encode_x_map(d, g, x, box_bytes, CU_TENSOR_MAP_SWIZZLE_NONE, &xm);
+    if (s != QC_OK) return s;
+    const int64_t PQ = static_cast<int64_t>(g.P) * g.Q;
+    const int img = static_cast<int>(m0 / PQ);
+    const int64_t rem = m0 - img * PQ;
+    const int p0 = static_cast<int>(rem / g.Q), q0 = static_cast<int>(rem % g.Q);
+    const uint32_t bytes = static_cast<uint32_t>(qc::kBM * box_bytes);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    cudaError_t e = cudaFuncSetAttribute(qc::qconv_debug_im2col_kernel,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+    if (e != cudaSuccess) return cuda_fail(e);
+    qc::qconv_debug_im2col_kernel<<<1, 128, bytes + 1024, st>>>(
+        xm, c_byte, q0 * d->stride_w - d->pad_w, p0 * d->stride_h - d->pad_h, img,
+        static_cast<uint16_t>(s_ * d->dil_w), static_cast<uint16_t>(r * d->dil_h), bytes,
+        static_cast<uint8_t *>(out));
+    e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e);
+    return QC_OK;
+}
+
+}  // extern "C"
