@@ -10,7 +10,7 @@
 //     channels (one UMMA tile, accumulator in TMEM), K-stage = one filter tap
 //     x BK bytes of channels.  Warp specialisation replaces the paper's warp
 //     tiling: warp 0 issues TMA, one thread of warp 1 issues tcgen05.mma,
-//     warps 4-7 run the epilogue, (4-bit) warps 8-11 widen int4 to int8.
+//     warps 4-11 run the epilogue, (4-bit) warps 12-15 widen int4 to int8.
 //   * register prefetch buffer -> a multi-stage shared-memory
 //     ring guarded by mbarriers; the epilogue of tile i overlaps the MMAs of
 //     tile i+1 through two TMEM accumulator buffers.
@@ -31,9 +31,9 @@ constexpr int kBM = 128;             // output pixels per tile (UMMA M)
 constexpr int kMaxBN = 256;
 constexpr int kWarpTMA = 0;
 constexpr int kWarpMMA = 1;
-constexpr int kWarpEpi0 = 4;         // warps 4..7: epilogue (TMEM lane quarters 0..3)
-constexpr int kNumEpiWarps = 4;
-constexpr int kWarpCvt0 = 8;         // warps 8..11: int4 -> int8 converters (4-bit only)
+constexpr int kWarpEpi0 = 4;         // warps 4..11: epilogue (TMEM lane quarter = warp % 4)
+constexpr int kNumEpiWarps = 8;
+constexpr int kWarpCvt0 = 12;        // warps 12..15: int4 -> int8 converters (4-bit only)
 constexpr int kNumCvtWarps = 4;
 
 enum OutKind { OUT_S32 = 0, OUT_U8 = 1, OUT_S8 = 2, OUT_U4 = 3, OUT_S4 = 4 };
@@ -58,54 +58,24 @@ struct ConvParams {
 };
 
 // ------------------------------------------------------------------ epilogue helpers
-// Per-column re-quantization constants (built once per N tile into smem):
-//   mode 0 (shift in [32,52]): t+zy = hi32(acc*m + C) >> (shift-32),
-//          C = bias*m + 2^(shift-1) + zy*2^shift   (exact)
-//   mode 1 (other shifts):     t = (acc*m + C) >> shift (int64), C = bias*m + 2^(shift-1)
-//   S32:                       y = acc + bias
-struct __align__(16) ColParam {
-    int32_t m;
-    int32_t shm;     // shift amount | mode << 8
-    int64_t c;
+// Per-column epilogue constants (16 B in smem).  Their meaning is chosen per
+// 32-column chunk (warp-uniform branch, no per-element branches):
+//   fast chunk  {b, m, rhi, sh}: 33 <= shift <= 52 for all 32 columns, x_zero == 0:
+//       v = acc + b (int32, exact by the API contract)
+//       y = clamp((mulhi(v, m) + rhi) >> sh),  rhi = 2^(n-33) + zy*2^(n-32), sh = n-32
+//     exact: v*m + 2^(n-1) + zy*2^n = v*m + rhi*2^32, so floor(./2^n) = (floor(v*m/2^32)+rhi)>>sh
+//   general chunk {b, m, n, 0}: t = (int64(v)*m + 2^(n-1)) >> n (int64), clamp, + zy
+//   S32 output   {b, 0, 0, 0}:  y = acc + b
+struct __align__(16) EpiCol {
+    int32_t b, m, c2, c3;
 };
 
-__device__ __forceinline__ ColParam make_col_param(const ConvParams &p, int k, bool s32) {
-    ColParam cp;
-    const int32_t b = (p.bias && k < p.K) ? __ldg(p.bias + k) : 0;
-    if (s32 || k >= p.K) {
-        cp.m = 0; cp.shm = 0; cp.c = b;
-        return cp;
-    }
-    const int32_t m = __ldg(p.mult + k);
-    const int32_t n = __ldg(p.shift + k);
-    const int64_t prod = static_cast<int64_t>(b) * m + (static_cast<int64_t>(1) << (n - 1));
-    cp.m = m;
-    if (n >= 32 && n <= 52) {
-        cp.c = prod + (static_cast<int64_t>(p.y_zero) << n);
-        cp.shm = n - 32;
-    } else {
-        cp.c = prod;
-        cp.shm = n | (1 << 8);
-    }
-    return cp;
-}
-
-template <int OUT>
-__device__ __forceinline__ int32_t requant_one(int32_t acc, const ColParam &cp, int32_t lo,
-                                               int32_t hi, int32_t zy) {
-    if (OUT == OUT_S32) return acc + static_cast<int32_t>(cp.c);
-    int32_t y;
-    if ((cp.shm >> 8) == 0) {
-        const int64_t prod = static_cast<int64_t>(acc) * cp.m + cp.c;   // mad.wide.s32
-        y = static_cast<int32_t>(prod >> 32) >> (cp.shm & 63);
-    } else {
-        const int64_t prod = static_cast<int64_t>(acc) * cp.m + cp.c;
-        int64_t t = prod >> (cp.shm & 63);
-        const int64_t lo64 = static_cast<int64_t>(lo) - zy, hi64 = static_cast<int64_t>(hi) - zy;
-        t = t < lo64 ? lo64 : (t > hi64 ? hi64 : t);
-        y = static_cast<int32_t>(t) + zy;
-    }
-    return min(hi, max(lo, y));
+__device__ __forceinline__ int4 lds128(uint32_t addr) {
+    int4 v;
+    asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                 : "r"(addr));
+    return v;
 }
 
 // number of valid filter taps along one spatial dim for output coordinate o:
@@ -123,87 +93,123 @@ __device__ __forceinline__ void valid_tap_range(int o, int stride, int pad, int 
     t1 = max(lo, hi);
 }
 
-// Process NC (16 or 32) accumulator columns of one output row and store them.
-template <int OUT, int NC>
-__device__ __forceinline__ void epilogue_chunk(const ConvParams &p, const uint32_t (&v)[32],
-                                               const ColParam *par, int col0, int n0, int64_t m,
-                                               bool row_ok, int zx_r0, int zx_r1, int zx_s0,
-                                               int zx_s1) {
-    int32_t yv[NC];
+// Fast chunk: 32 columns, all constants from smem (broadcast LDS.128), no branches.
+template <int H>
+__device__ __forceinline__ void epi_fast16(uint32_t (&v)[32], uint32_t par_addr, int32_t lo,
+                                           int32_t hi) {
 #pragma unroll
-    for (int j = 0; j < NC; ++j) {
-        int32_t acc = static_cast<int32_t>(v[j]);
-        if (p.x_zero != 0) {
-            const int k = n0 + col0 + j;
-            if (k < p.K) {
-                const int RS1 = p.S + 1;
-                const int32_t *t = p.zx_table + static_cast<int64_t>(k) * (p.R + 1) * RS1;
-                const int32_t rect = __ldg(t + zx_r1 * RS1 + zx_s1) - __ldg(t + zx_r0 * RS1 + zx_s1) -
-                                     __ldg(t + zx_r1 * RS1 + zx_s0) + __ldg(t + zx_r0 * RS1 + zx_s0);
-                acc -= p.x_zero * rect;
-            }
-        }
-        const ColParam cp = par[col0 + j];
-        yv[j] = requant_one<OUT>(acc, cp, p.clamp_lo, p.clamp_hi, p.y_zero);
+    for (int j = H; j < H + 16; ++j) {
+        const int4 pr = lds128(par_addr + 16u * j);
+        const int32_t x = static_cast<int32_t>(v[j]) + pr.x;
+        const int32_t t = (__mulhi(x, pr.y) + pr.z) >> pr.w;
+        v[j] = static_cast<uint32_t>(min(hi, max(lo, t)));
     }
-    if (!row_ok) return;
-    const int kc = n0 + col0;                    // first output channel of the chunk
-    const bool in_range = kc + NC <= p.K;
-    if (OUT == OUT_S32) {
-        int32_t *dst = reinterpret_cast<int32_t *>(static_cast<uint8_t *>(p.y) + m * p.y_row_bytes) + kc;
-        if (in_range && (reinterpret_cast<uintptr_t>(dst) & 15u) == 0) {
+}
+
+// General chunk (any shift, optional x_zero border correction, or int32 output).
+template <int OUT, bool ZX, int H>
+__device__ __forceinline__ void epi_general16(const ConvParams &p, uint32_t (&v)[32],
+                                              uint32_t par_addr, int kc, int zr0, int zr1,
+                                              int zs0, int zs1) {
 #pragma unroll
-            for (int j = 0; j < NC; j += 4) st_global_v4(dst + j, yv[j], yv[j + 1], yv[j + 2], yv[j + 3]);
+    for (int j = H; j < H + 16; ++j) {
+        const int4 pr = lds128(par_addr + 16u * j);
+        int32_t x = static_cast<int32_t>(v[j]) + pr.x;
+        if (ZX) {
+            const int k = min(kc + j, p.K - 1);
+            const int RS1 = p.S + 1;
+            const int32_t *t = p.zx_table + static_cast<int64_t>(k) * (p.R + 1) * RS1;
+            const int32_t rect = __ldg(t + zr1 * RS1 + zs1) - __ldg(t + zr0 * RS1 + zs1) -
+                                 __ldg(t + zr1 * RS1 + zs0) + __ldg(t + zr0 * RS1 + zs0);
+            x -= p.x_zero * rect;
+        }
+        if (OUT == OUT_S32) {
+            v[j] = static_cast<uint32_t>(x);
         } else {
-            for (int j = 0; j < NC && kc + j < p.K; ++j) dst[j] = yv[j];
-        }
-    } else if (OUT == OUT_U8 || OUT == OUT_S8) {
-        uint32_t w[NC / 4];
-#pragma unroll
-        for (int j = 0; j < NC / 4; ++j) {
-            if (OUT == OUT_U8)
-                w[j] = pack_sat_u8(yv[4 * j + 1], yv[4 * j], pack_sat_u8(yv[4 * j + 3], yv[4 * j + 2], 0u));
-            else
-                w[j] = pack_sat_s8(yv[4 * j + 1], yv[4 * j], pack_sat_s8(yv[4 * j + 3], yv[4 * j + 2], 0u));
-        }
-        uint8_t *dst = static_cast<uint8_t *>(p.y) + m * p.y_row_bytes + kc;
-        if (in_range && (reinterpret_cast<uintptr_t>(dst) & 15u) == 0) {
-#pragma unroll
-            for (int j = 0; j < NC / 4; j += 4) st_global_v4(dst + 4 * j, w[j], w[j + 1], w[j + 2], w[j + 3]);
-        } else {
-            for (int j = 0; j < NC && kc + j < p.K; ++j) dst[j] = static_cast<uint8_t>(w[j >> 2] >> (8 * (j & 3)));
-        }
-    } else {
-        uint32_t w[NC / 8];
-#pragma unroll
-        for (int j = 0; j < NC / 8; ++j) {
-            const int b = 8 * j;
-            if (OUT == OUT_U4) {
-                uint32_t t = pack_sat_u4(yv[b + 7], yv[b + 6], 0u);
-                t = pack_sat_u4(yv[b + 5], yv[b + 4], t);
-                t = pack_sat_u4(yv[b + 3], yv[b + 2], t);
-                w[j] = pack_sat_u4(yv[b + 1], yv[b], t);
-            } else {
-                uint32_t t = pack_sat_s4(yv[b + 7], yv[b + 6], 0u);
-                t = pack_sat_s4(yv[b + 5], yv[b + 4], t);
-                t = pack_sat_s4(yv[b + 3], yv[b + 2], t);
-                w[j] = pack_sat_s4(yv[b + 1], yv[b], t);
-            }
-        }
-        uint8_t *dst = static_cast<uint8_t *>(p.y) + m * p.y_row_bytes + kc / 2;
-        if (in_range && (reinterpret_cast<uintptr_t>(dst) & (NC == 32 ? 15u : 7u)) == 0) {
-            if (NC == 32) st_global_v4(dst, w[0], w[1], w[2], w[3]);
-            else *reinterpret_cast<uint2 *>(dst) = make_uint2(w[0], w[1]);
-        } else {
-            for (int j = 0; 2 * j < NC && kc + 2 * j < p.K; ++j)
-                dst[j] = static_cast<uint8_t>(w[j >> 2] >> (8 * (j & 3)));
+            const int64_t prod = static_cast<int64_t>(x) * pr.y + (static_cast<int64_t>(1) << (pr.z - 1));
+            int64_t t = prod >> pr.z;
+            const int64_t lo64 = static_cast<int64_t>(p.clamp_lo) - p.y_zero;
+            const int64_t hi64 = static_cast<int64_t>(p.clamp_hi) - p.y_zero;
+            t = t < lo64 ? lo64 : (t > hi64 ? hi64 : t);
+            v[j] = static_cast<uint32_t>(static_cast<int32_t>(t) + p.y_zero);
         }
     }
 }
 
+// Pack and store outputs v[H .. H+16) of one row = output channels [kc, kc+16).
+template <int OUT, int H>
+__device__ __forceinline__ void store16(const ConvParams &p, const uint32_t (&v)[32], int kc,
+                                        int64_t m) {
+    uint8_t *rowp = static_cast<uint8_t *>(p.y) + m * p.y_row_bytes;
+    const bool in_range = kc + 16 <= p.K;
+    if (OUT == OUT_S32) {
+        uint32_t *dst = reinterpret_cast<uint32_t *>(rowp) + kc;
+        if (in_range && (reinterpret_cast<uintptr_t>(dst) & 15u) == 0) {
+#pragma unroll
+            for (int j = 0; j < 16; j += 4) st_global_v4(dst + j, v[H + j], v[H + j + 1], v[H + j + 2], v[H + j + 3]);
+        } else {
+#pragma unroll
+            for (int j = 0; j < 16; ++j)
+                if (kc + j < p.K) dst[j] = v[H + j];
+        }
+    } else if (OUT == OUT_U8 || OUT == OUT_S8) {
+        uint32_t w[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int32_t *y = reinterpret_cast<const int32_t *>(&v[H + 4 * j]);
+            if (OUT == OUT_U8)
+                w[j] = pack_sat_u8(y[1], y[0], pack_sat_u8(y[3], y[2], 0u));
+            else
+                w[j] = pack_sat_s8(y[1], y[0], pack_sat_s8(y[3], y[2], 0u));
+        }
+        uint8_t *dst = rowp + kc;
+        if (in_range && (reinterpret_cast<uintptr_t>(dst) & 15u) == 0) {
+            st_global_v4(dst, w[0], w[1], w[2], w[3]);
+        } else {
+#pragma unroll
+            for (int j = 0; j < 16; ++j)
+                if (kc + j < p.K) dst[j] = static_cast<uint8_t>(w[j >> 2] >> (8 * (j & 3)));
+        }
+    } else {
+        uint32_t w[2];
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+            const int32_t *y = reinterpret_cast<const int32_t *>(&v[H + 8 * j]);
+            if (OUT == OUT_U4) {
+                uint32_t t = pack_sat_u4(y[7], y[6], 0u);
+                t = pack_sat_u4(y[5], y[4], t);
+                t = pack_sat_u4(y[3], y[2], t);
+                w[j] = pack_sat_u4(y[1], y[0], t);
+            } else {
+                uint32_t t = pack_sat_s4(y[7], y[6], 0u);
+                t = pack_sat_s4(y[5], y[4], t);
+                t = pack_sat_s4(y[3], y[2], t);
+                w[j] = pack_sat_s4(y[1], y[0], t);
+            }
+        }
+        uint8_t *dst = rowp + kc / 2;
+        if (in_range && (reinterpret_cast<uintptr_t>(dst) & 7u) == 0) {
+            asm volatile("st.global.v2.b32 [%0], {%1, %2};" ::"l"(dst), "r"(w[0]), "r"(w[1]) : "memory");
+        } else {
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+                if (kc + 2 * j < p.K) dst[j] = static_cast<uint8_t>(w[j >> 2] >> (8 * (j & 3)));
+        }
+    }
+}
+
+template <int OUT, bool ZX, int H>
+__device__ __forceinline__ void epi_half(const ConvParams &p, uint32_t (&v)[32], uint32_t pa,
+                                         bool fast, int kc, int64_t m, bool row_ok, int zr0,
+                                         int zr1, int zs0, int zs1) {
+    if (fast) epi_fast16<H>(v, pa, p.clamp_lo, p.clamp_hi);
+    else epi_general16<OUT, ZX, H>(p, v, pa, kc - H, zr0, zr1, zs0, zs1);
+    if (row_ok) store16<OUT, H>(p, v, kc, m);
+}
+
 // ------------------------------------------------------------------ the kernel
-template <bool IS4, int OUT>
-__global__ void __launch_bounds__(IS4 ? 384 : 256, 1)
+template <bool IS4, int OUT, bool ZX>
+__global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
 qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap wmap,
                  const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -220,7 +226,8 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
     uint64_t *tfull = bars + 3 * NS;        // [2]  MMA -> epilogue
     uint64_t *tempty = bars + 3 * NS + 2;   // [2]  epilogue -> MMA
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 4);
-    ColParam *par = reinterpret_cast<ColParam *>(smem + p.off_par);
+    EpiCol *par = reinterpret_cast<EpiCol *>(smem + p.off_par);
+    uint8_t *chunk_fast = smem + p.off_par + 16 * kMaxBN;   // [8] per 32-column chunk
 
     if (warp == kWarpTMA && lane == 0) {
         tma_prefetch_desc(&xmap);
@@ -307,10 +314,14 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
             }
         }
     } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kNumEpiWarps) {
-        // ===================== epilogue (4 warps, one TMEM lane quarter each) =====================
-        const int quarter = warp & 3;
+        // ===================== epilogue (8 warps: lane quarter = warp%4, column half) ============
+        const int ew = warp - kWarpEpi0;                 // 0..7
+        const int quarter = warp & 3;                    // TMEM lanes 32*quarter .. +31
+        const int half = ew >> 2;                        // which 32-column chunks
         const int row = quarter * 32 + lane;
-        const int et = (warp - kWarpEpi0) * 32 + lane;     // 0..127
+        const uint32_t par_base = smem_u32(par);
+        const int nchunks = (p.BN + 31) / 32;
+        const bool force_general = (OUT == OUT_S32) || ZX;
         int cached_n0 = -1;
         int it = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
@@ -319,16 +330,37 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
             const int m0 = (tile / p.n_tiles_n) * kBM;
             const int n0 = (tile % p.n_tiles_n) * p.BN;
             if (n0 != cached_n0) {
+                // per-column constants for this N tile; thread (ew, lane) owns column 32*ew+lane
                 named_bar_sync(1, kNumEpiWarps * 32);
-                for (int c = et; c < p.BN; c += kNumEpiWarps * 32)
-                    par[c] = make_col_param(p, n0 + c, OUT == OUT_S32);
+                const int c = ew * 32 + lane;
+                const int k = n0 + c;
+                EpiCol e;
+                e.b = (p.bias && k < p.K) ? __ldg(p.bias + k) : 0;
+                e.m = 0; e.c2 = 0; e.c3 = 0;
+                int32_t nn = 40;
+                if (OUT != OUT_S32 && k < p.K) {
+                    e.m = __ldg(p.mult + k);
+                    nn = __ldg(p.shift + k);
+                }
+                const bool fast = !force_general &&
+                                  __ballot_sync(0xffffffffu, nn >= 33 && nn <= 52) == 0xffffffffu;
+                if (OUT != OUT_S32 && k < p.K) {
+                    if (fast) {
+                        e.c2 = (1 << (nn - 33)) + p.y_zero * (1 << (nn - 32));
+                        e.c3 = nn - 32;
+                    } else {
+                        e.c2 = nn;
+                    }
+                }
+                if (c < p.BN) *reinterpret_cast<EpiCol *>(reinterpret_cast<uint8_t *>(par) + 16 * c) = e;
+                if (lane == 0) chunk_fast[ew] = fast ? 1 : 0;
                 named_bar_sync(1, kNumEpiWarps * 32);
                 cached_n0 = n0;
             }
             const int64_t m = static_cast<int64_t>(m0) + row;
             const bool row_ok = m < p.M;
             int zr0 = 0, zr1 = 0, zs0 = 0, zs1 = 0;
-            if (p.x_zero != 0) {
+            if (ZX) {
                 const int mm = row_ok ? static_cast<int>(m) : 0;
                 const int rem = mm % p.PQ;
                 const int pp = rem / p.Q;
@@ -341,18 +373,18 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
             const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
                                    static_cast<uint32_t>(buf * p.BN);
             uint32_t v[32];
-            int col0 = 0;
-            for (; col0 + 32 <= p.BN; col0 += 32) {
+            for (int ci = half; ci < nchunks; ci += 2) {
+                const int col0 = ci * 32;
+                const int nc = min(32, p.BN - col0);
                 __syncwarp();
-                tmem_ld_32x32b_x32(taddr + col0, v);
+                if (nc == 32) tmem_ld_32x32b_x32(taddr + col0, v);
+                else tmem_ld_32x32b_x16(taddr + col0, v);
                 tmem_wait_ld();
-                epilogue_chunk<OUT, 32>(p, v, par, col0, n0, m, row_ok, zr0, zr1, zs0, zs1);
-            }
-            if (col0 < p.BN) {
-                __syncwarp();
-                tmem_ld_32x32b_x16(taddr + col0, v);
-                tmem_wait_ld();
-                epilogue_chunk<OUT, 16>(p, v, par, col0, n0, m, row_ok, zr0, zr1, zs0, zs1);
+                const uint32_t pa = par_base + 16u * col0;
+                const bool fast = !force_general && chunk_fast[ci];
+                epi_half<OUT, ZX, 0>(p, v, pa, fast, n0 + col0, m, row_ok, zr0, zr1, zs0, zs1);
+                if (nc == 32)
+                    epi_half<OUT, ZX, 16>(p, v, pa, fast, n0 + col0 + 16, m, row_ok, zr0, zr1, zs0, zs1);
             }
             tc_fence_before();
             __syncwarp();

@@ -65,8 +65,19 @@ __global__ void __launch_bounds__(256) quantize_pack_kernel(const __grid_constan
                     q[4 * j + 3] = quantize_one(v.w, p);
                 }
             }
-        } else {
+        } else if (p.c_pad % 16 == 0) {
+            // one group = 16 channels of one pixel: a single division per group
+            const int32_t gpp = p.c_pad / 16;
+            const int64_t pix = g / gpp;
+            const int32_t ch0 = static_cast<int32_t>(g - pix * gpp) * 16;
+            const int64_t base = pix * p.c;
 #pragma unroll
+            for (int j = 0; j < 16; ++j) {
+                const int32_t ch = ch0 + j;
+                q[j] = ch < p.c ? quantize_one(load_x(p, base + ch), p) : p.z;
+            }
+        } else {
+#pragma unroll 1
             for (int j = 0; j < 16; ++j) {
                 const int64_t e = e0 + j;
                 if (e < total) {

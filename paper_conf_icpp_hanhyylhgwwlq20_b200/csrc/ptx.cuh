@@ -54,15 +54,14 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
     return t;
 }
-// Wait for the phase with the given parity to complete.  A wait longer than
-// ~4 s traps (turns a protocol bug into a reported launch error, not a hang).
+// Wait for the phase with the given parity to complete.  try_wait suspends the
+// thread for a hardware-chosen interval per call; ~2^26 unsuccessful polls
+// (seconds) trap, turning a protocol bug into a launch error instead of a hang.
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     const uint32_t a = smem_u32(bar);
-    if (mbar_try_wait(a, parity)) return;
-    const uint64_t t0 = globaltimer_ns();
     uint32_t it = 0;
     while (!mbar_try_wait(a, parity)) {
-        if ((++it & 1023u) == 0 && globaltimer_ns() - t0 > 4000000000ull) __trap();
+        if (++it == (1u << 26)) __trap();
     }
 }
 

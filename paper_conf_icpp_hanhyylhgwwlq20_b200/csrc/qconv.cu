@@ -217,7 +217,7 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const uint32_t b_bytes = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * pl->BK, 1024));
     const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(qc::kBM * pl->bkp) : 0u;
     const uint32_t per_stage = a_bytes + b_bytes + stg_bytes;
-    const uint32_t fixed = static_cast<uint32_t>(BN) * 16u + 1024u;     // params + barriers
+    const uint32_t fixed = static_cast<uint32_t>(qc::kMaxBN) * 16u + 64u + 1024u;  // params, flags, barriers
     const uint32_t budget = 227u * 1024u - 1024u - fixed;
     int stages = static_cast<int>(budget / per_stage);
     stages = std::min(stages, 8);
@@ -229,11 +229,11 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.off_b = p.off_a + a_bytes * stages;
     p.off_stg = p.off_b + b_bytes * stages;
     p.off_par = static_cast<uint32_t>(align_up(p.off_stg + stg_bytes * stages, 16));
-    p.off_bar = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(BN) * 16u, 8));
+    p.off_bar = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 64u, 8));
     const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 4) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;       // + alignment slack for the 1024-B base
     pl->grid = std::min(pl->num_tiles, sms);
-    pl->threads = is4 ? 384 : 256;
+    pl->threads = is4 ? 512 : 384;
     p.a_stage_bytes = a_bytes;
     p.b_stage_bytes = b_bytes;
     p.stg_stage_bytes = stg_bytes;
@@ -315,10 +315,10 @@ qc_status encode_w_map(const qconv_desc *d, const Geometry &g, const void *w8, i
     return QC_OK;
 }
 
-template <bool IS4, int OUT>
-qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
-                      cudaStream_t stream) {
-    auto kern = qc::qconv_fwd_kernel<IS4, OUT>;
+template <bool IS4, int OUT, bool ZX>
+qc_status launch_conv_t(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
+                        cudaStream_t stream) {
+    auto kern = qc::qconv_fwd_kernel<IS4, OUT, ZX>;
     static int configured_smem = 0;   // per instantiation; max over calls is safe to keep
     if (configured_smem < static_cast<int>(pl.smem_bytes)) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -337,6 +337,13 @@ qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, pl.cp);
     if (e != cudaSuccess) return cuda_fail(e);
     return QC_OK;
+}
+
+template <bool IS4, int OUT>
+qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
+                      cudaStream_t stream) {
+    return pl.cp.x_zero != 0 ? launch_conv_t<IS4, OUT, true>(pl, xm, wm, stream)
+                             : launch_conv_t<IS4, OUT, false>(pl, xm, wm, stream);
 }
 
 }  // namespace

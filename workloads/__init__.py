@@ -263,6 +263,64 @@ def make_layer_inputs(cs: ConvShape, bits: int, seed: int, *, out_bits: Optional
                        clamp_hi=int(hi), s_x=float(s_x), s_w=s_w, s_y=float(s_y), relu=relu)
 
 
+@dataclasses.dataclass
+class LayerParams:
+    """Weights and scales of one layer (no activations) -- for the bench trunk."""
+    shape: ConvShape
+    x_t: int
+    w_t: int
+    y_t: int
+    w_codes: np.ndarray
+    w_bytes: np.ndarray
+    bias: np.ndarray
+    s_x: float
+    s_w: np.ndarray
+    s_y: float
+    clamp_lo: int
+    clamp_hi: int
+    c_store: int
+
+
+def make_layer_params(cs: ConvShape, bits: int, seed: int, *, c_store: Optional[int] = None,
+                      relu: bool = True) -> LayerParams:
+    """Seeded weights/bias/scales with the same recipe as make_layer_inputs; the output
+    scale uses the expected second moment of post-ReLU half-normal activation codes."""
+    rng = np.random.default_rng(seed)
+    x_t = U4 if bits == 4 else U8
+    w_t = S4 if bits == 4 else S8
+    y_t = x_t
+    c_st = cs.c if c_store is None else c_store
+    w_codes, s_w = symmetric_weight_codes(rng, cs.k, (cs.r, cs.s, cs.c), bits)
+    bias = rng.integers(-(1 << 12), (1 << 12) + 1, size=cs.k).astype(np.int32)
+    if bits == 4:
+        bias = (bias // 64).astype(np.int32)
+    if c_st != cs.c:
+        wp = np.zeros((cs.k, cs.r, cs.s, c_st), dtype=np.int64)
+        wp[..., :cs.c] = w_codes
+        w_codes = wp
+    qx_max = (1 << bits) - 1
+    sig = 40 / 255 * qx_max
+    ex2 = 0.5 * sig * sig
+    ew2 = float(np.mean(w_codes[..., :cs.c].astype(np.float64) ** 2))
+    sigma_acc = np.sqrt(cs.r * cs.s * cs.c * ex2 * ew2) + 1.0
+    s_x = np.float32(0.05)
+    s_y = np.float32(float(s_x) * float(np.median(s_w)) * 2.33 * sigma_acc / DTYPE_RANGE[y_t][1])
+    lo, hi = DTYPE_RANGE[y_t]
+    return LayerParams(shape=cs, x_t=x_t, w_t=w_t, y_t=y_t, w_codes=w_codes,
+                       w_bytes=pack_codes(w_codes, w_t), bias=bias, s_x=float(s_x), s_w=s_w,
+                       s_y=float(s_y), clamp_lo=max(lo, 0) if relu else lo, clamp_hi=hi,
+                       c_store=c_st)
+
+
+def post_relu_codes_fast(rng: np.random.Generator, shape, bits: int) -> np.ndarray:
+    """uint8 post-ReLU codes (same distribution as post_relu_codes, less memory)."""
+    qmax = (1 << bits) - 1
+    v = np.abs(rng.standard_normal(size=shape, dtype=np.float32)) * np.float32(40 / 255 * qmax)
+    v = np.rint(v)
+    v[rng.random(size=shape, dtype=np.float32) < 0.5] = 0
+    return np.clip(v, 0, qmax).astype(np.uint8)
+
+
 def stored_channels(cs: ConvShape, bits: int) -> int:
     """Stored channel count the library accepts for this layer (C padded to a
     multiple of 32 elements only where the real C is smaller, i.e. the stem)."""
