@@ -100,13 +100,16 @@ class Trunk:
         # ---- weights + params: generated on rank 0, broadcast once (the only collective)
         params = []
         for cs, c_st, i in specs:
+            stem = i == 0
             if rank0:
-                lp = W.make_layer_params(cs, bits, W.layer_seed(i), c_store=c_st)
-                wb = torch.from_numpy(np.ascontiguousarray(lp.w_bytes).reshape(-1)).to(device)
+                lp = W.make_layer_params(cs, bits, W.layer_seed(i), c_store=None if stem else c_st)
+                # stem: C = 3 codes stored one per byte (space-to-depth path)
+                wbytes = W.pack_codes(lp.w_codes, W.S8) if stem else lp.w_bytes
+                wb = torch.from_numpy(np.ascontiguousarray(wbytes).reshape(-1)).to(device)
                 m, n = qc.qconv_requant_params(lp.s_x, lp.s_w, lp.s_y)
                 pb = torch.from_numpy(np.stack([lp.bias, m, n]).astype(np.int32)).to(device)
             else:
-                nbytes = cs.k * cs.r * cs.s * c_st * bits // 8
+                nbytes = cs.k * cs.r * cs.s * (cs.c if stem else c_st * bits // 8)
                 wb = torch.empty(nbytes, dtype=torch.uint8, device=device)
                 pb = torch.empty((3, cs.k), dtype=torch.int32, device=device)
             if dist_ctx is not None and dist_ctx["world"] > 1:
@@ -117,12 +120,15 @@ class Trunk:
         rank = 0 if dist_ctx is None else dist_ctx["rank"]
         g.manual_seed(W.SEED_BASE + 7919 * rank)
         stem = specs[0][0]
-        self.stem_c_pad = specs[0][1]
         self.x_float = torch.relu(torch.randn((batch, stem.h, stem.w, stem.c), generator=g,
                                               device=device, dtype=torch.float32))
         self.s_in = 3.0 / 15 if bits == 4 else 3.0 / 255
-        self.x_q = torch.empty((batch, stem.h, stem.w, self.stem_c_pad * bits // 8),
-                               dtype=torch.uint8, device=device)
+        # the stem (7x7/s2, C=3) runs in space-to-depth form: 4x4/s1 over C=16 byte codes
+        self.stem_desc = qc.make_desc(batch, stem.h, stem.w, stem.c, stem.k, stem.r, stem.s,
+                                      stride=stem.stride, pad=stem.pad, x_t=x_t, w_t=W.S8,
+                                      y_t=x_t, relu=True)
+        d2 = qc.qconv_s2d_desc(self.stem_desc)
+        self.x_q = torch.empty((d2.n, d2.h, d2.w, d2.c), dtype=torch.uint8, device=device)
         # res2 input: max-pool is outside the method -> separately drawn codes
         rng = np.random.default_rng(W.SEED_BASE + 31 * rank + 1)
         codes = W.post_relu_codes_fast(rng, (batch, 56, 56, 64), bits)
@@ -134,10 +140,14 @@ class Trunk:
         cur = None
         block_in = None
         for (cs, c_st, i), (wb, pb) in zip(specs, params):
-            d = qc.make_desc(cs.n, cs.h, cs.w, c_st, cs.k, cs.r, cs.s, stride=cs.stride,
-                             pad=cs.pad, x_t=x_t, w_t=w_t, y_t=x_t, relu=True)
-            w_prep = qc.qconv_prepare_weights(d, wb)
-            d.w_prepared = 1
+            if i == 0:
+                w_prep = qc.qconv_prepare_weights_s2d(self.stem_desc, wb)
+                d = qc.qconv_s2d_desc(self.stem_desc)
+            else:
+                d = qc.make_desc(cs.n, cs.h, cs.w, c_st, cs.k, cs.r, cs.s, stride=cs.stride,
+                                 pad=cs.pad, x_t=x_t, w_t=w_t, y_t=x_t, relu=True)
+                w_prep = qc.qconv_prepare_weights(d, wb)
+                d.w_prepared = 1
             p, q = qc.out_hw(d)
             y = torch.empty((cs.n, p, q, cs.k * bits // 8), dtype=torch.uint8, device=device)
             role = W.RESNET50_LAYERS[i]["role"]
@@ -153,7 +163,7 @@ class Trunk:
                 src = block_in
             else:
                 src = cur
-            assert src.shape[1] == cs.h and src.shape[2] == cs.w, cs.name
+            assert src.shape[1] == d.h and src.shape[2] == d.w, cs.name
             ops, nbytes = layer_algorithmic(cs, bits)
             self.layers.append(dict(name=cs.name, desc=d, w=w_prep, bias=pb[0], m=pb[1],
                                     n=pb[2], x=src, y=y, ops=ops, bytes=nbytes))
@@ -167,10 +177,14 @@ class Trunk:
         return sum(L["ops"] for L in self.layers)
 
     @property
+    def quantize_bytes(self):
+        """Algorithmic bytes of the stem quantization: fp32 read + space-to-depth codes written."""
+        d, x = self.stem_desc, self.x_q
+        return d.n * d.h * d.w * d.c * 4 + x.numel()
+
+    @property
     def bytes_per_step(self):
-        stem = self.layers[0]["desc"]
-        qbytes = self.batch * stem.h * stem.w * (4 * 3 + self.stem_c_pad * self.bits / 8)
-        return sum(L["bytes"] for L in self.layers) + qbytes
+        return sum(L["bytes"] for L in self.layers) + self.quantize_bytes
 
     def launches_per_step(self):
         return 1 + len(self.layers)
@@ -178,8 +192,8 @@ class Trunk:
     def step(self, events=None, x_float=None):
         """Enqueue one step on the current stream; events[i] recorded after launch i."""
         qc = self.qc
-        qc.qconv_quantize_pack(self.x_float if x_float is None else x_float, self.s_in, 0,
-                               self.x_t, c_pad=self.stem_c_pad, out=self.x_q)
+        qc.qconv_quantize_pack_s2d(self.stem_desc, self.x_float if x_float is None else x_float,
+                                   self.s_in, out=self.x_q)
         if events is not None:
             events[0].record()
         for j, L in enumerate(self.layers):
@@ -256,6 +270,7 @@ class OracleTrunk:
         os.environ.setdefault("OMP_NUM_THREADS", str(self.cores))
         self.specs = trunk_layers(bits, 1)
         self.x_t = W.U4 if bits == 4 else W.U8
+        self.specs = [(cs, 4 if i == 0 else c_st, i) for cs, c_st, i in self.specs]
         self.lps = [W.make_layer_params(cs, bits, W.layer_seed(i), c_store=c_st)
                     for cs, c_st, i in self.specs]
         self.mns = [oracle.requant_params(lp.s_x, lp.s_w, lp.s_y) for lp in self.lps]
@@ -514,8 +529,10 @@ def main():
                          "conv_share_of_step": conv_total_ms / ms_per_step,
                          "algorithmic_ops_per_step": float(conv_ops.sum()),
                          "algorithmic_bytes_per_step": float(conv_bytes.sum())},
-            "quantize_pack": {"us": q_ms * 1e3,
-                              "gbs": (trunk.bytes_per_step - conv_bytes.sum()) / (q_ms / 1e3) / 1e9},
+            "quantize_pack": {"kernel": "quantize_s2d_kernel (fp32 -> space-to-depth codes)",
+                              "us": q_ms * 1e3,
+                              "gbs": trunk.quantize_bytes / (q_ms / 1e3) / 1e9,
+                              "frac_hbm": trunk.quantize_bytes / (q_ms / 1e3) / 1e9 / peaks["hbm_gbs"]},
             "e2e": e2e, "cpu_baseline": cpu, "clocks": clocks,
             "gpu_launches": args.steps * nL,
         }

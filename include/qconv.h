@@ -135,13 +135,39 @@ size_t qconv2d_workspace_size(const qconv_desc *d);
  *   multiplier, shift   device int32 [k]; may be NULL only for y_t == S32
  *   y          device, NHWC [n,p,q,k] packed y_t
  *   workspace  device, >= qconv2d_workspace_size(d) bytes (NULL if 0)
- * Errors: INVALID_ARG, UNSUPPORTED (mixed bit widths; c not a multiple of 32;
+ * Errors: INVALID_ARG, UNSUPPORTED (mixed bit widths; c not a multiple of 32 (8-bit
+ * c = 16 is accepted: two filter taps per 32-byte K step);
  * 4-bit y_t with odd k; pad/dilation beyond the TMA im2col corner range;
  * stride > 8), OVERFLOW_RISK, MISALIGNED, WORKSPACE, CUDA.
  */
 qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w,
                           const int32_t *bias, const int32_t *multiplier, const int32_t *shift,
                           void *y, void *workspace, size_t ws_bytes, void *stream);
+
+/*
+ * Space-to-depth form of a stride-2 convolution (the ResNet/VGG C=3 stem).  For a
+ * descriptor with stride 2 and dilation 1 (e.g. 7x7/s2/p3 over C=3), the 2x2
+ * space-to-depth rearrangement
+ *   X2[n,i,j,(2b+b')*c+cc] = code(x[n, 2i+b-pad_h, 2j+b'-pad_w, cc])  (x_zero where outside)
+ *   W2[k,a,a',(2b+b')*c+cc] = w[k, 2a+b, 2a'+b', cc]                  (0 beyond r, s)
+ * turns it into a stride-1, unpadded ceil(r/2) x ceil(s/2) convolution over C2 = 16
+ * (4c <= 16) or round_up(4c, 32) channels whose output is identical, byte for byte, to
+ * the original's (the same products, regrouped; P:L80's GEMM view with a denser K).
+ * Codes are stored one per byte (4-bit codes sign/zero-extended) so C2 = 16 meets the
+ * 16-byte TMA stride rule; the K reduction shrinks from r*s*round_up(c,32) to 16*C2.
+ *   qconv_s2d_desc          -> the transformed descriptor (x_t/w_t = byte containers,
+ *                              w_prepared = 1); pass it to qconv2d_forward
+ *   qconv_quantize_pack_s2d -> fused quantization (Z4, zero point d->x_zero, code range
+ *                              of d->x_t) + rearrangement of fp32/bf16 NHWC x into X2
+ *                              (device, qconv_s2d_desc(d).{n,h,w,c} bytes)
+ *   qconv_prepare_weights_s2d -> W2 (device int8, qconv_prepared_weight_bytes_s2d bytes)
+ * Errors: INVALID_ARG, UNSUPPORTED (stride != 2 or dilation != 1), MISALIGNED, CUDA.
+ */
+qc_status qconv_s2d_desc(const qconv_desc *d, qconv_desc *out);
+qc_status qconv_quantize_pack_s2d(const qconv_desc *d, const void *x, qc_ftype xt, float scale,
+                                  void *y, void *stream);
+size_t qconv_prepared_weight_bytes_s2d(const qconv_desc *d);
+qc_status qconv_prepare_weights_s2d(const qconv_desc *d, const void *w, void *w_prep, void *stream);
 
 /* Human-readable status; static storage, never NULL. */
 const char *qconv_status_string(qc_status s);

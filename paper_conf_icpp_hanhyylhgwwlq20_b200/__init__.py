@@ -74,6 +74,14 @@ def _lib():
         L.qconv2d_workspace_size.restype = sz
         L.qconv2d_forward.argtypes = [dp, vp, vp, vp, vp, vp, vp, vp, sz, vp]
         L.qconv2d_forward.restype = i32
+        L.qconv_s2d_desc.argtypes = [dp, dp]
+        L.qconv_s2d_desc.restype = i32
+        L.qconv_quantize_pack_s2d.argtypes = [dp, vp, i32, f32, vp, vp]
+        L.qconv_quantize_pack_s2d.restype = i32
+        L.qconv_prepared_weight_bytes_s2d.argtypes = [dp]
+        L.qconv_prepared_weight_bytes_s2d.restype = sz
+        L.qconv_prepare_weights_s2d.argtypes = [dp, vp, vp, vp]
+        L.qconv_prepare_weights_s2d.restype = i32
         L.qconv_debug_im2col_tile.argtypes = [dp, vp, i64, i32, i32, i32, i32, vp, vp]
         L.qconv_debug_im2col_tile.restype = i32
         _L = L
@@ -200,6 +208,38 @@ def qconv2d_forward(d: qconv_desc, x, w, bias=None, multiplier=None, shift=None,
     return y
 
 
+def qconv_s2d_desc(d: qconv_desc) -> qconv_desc:
+    """Descriptor of the space-to-depth form of a stride-2 conv (include/qconv.h)."""
+    o = qconv_desc()
+    _check("qconv_s2d_desc", _lib().qconv_s2d_desc(ctypes.byref(d), ctypes.byref(o)))
+    return o
+
+
+def qconv_quantize_pack_s2d(d: qconv_desc, x, scale: float, out=None, stream=None):
+    """fp32/bf16 NHWC x of the original conv -> X2 byte codes [n, h2, w2, c2]."""
+    import torch
+    assert x.is_cuda and x.is_contiguous() and x.dtype in (torch.float32, torch.bfloat16)
+    o = qconv_s2d_desc(d)
+    if out is None:
+        out = torch.empty((o.n, o.h, o.w, o.c), dtype=torch.uint8, device=x.device)
+    _check("qconv_quantize_pack_s2d", _lib().qconv_quantize_pack_s2d(
+        ctypes.byref(d), _ptr(x), QC_BF16 if x.dtype == torch.bfloat16 else QC_F32, float(scale),
+        _ptr(out), _stream(stream)))
+    return out
+
+
+def qconv_prepare_weights_s2d(d: qconv_desc, w, out=None, stream=None):
+    import torch
+    nb = int(_lib().qconv_prepared_weight_bytes_s2d(ctypes.byref(d)))
+    if nb == 0:
+        raise QConvError("qconv_prepare_weights_s2d", 2)
+    if out is None:
+        out = torch.empty(nb, dtype=torch.uint8, device=w.device)
+    _check("qconv_prepare_weights_s2d", _lib().qconv_prepare_weights_s2d(
+        ctypes.byref(d), _ptr(w), _ptr(out), _stream(stream)))
+    return out
+
+
 def qconv_debug_im2col_tile(d: qconv_desc, x, m0: int, r: int, s: int, c_byte: int,
                             box_bytes: int, stream=None):
     import torch
@@ -243,6 +283,7 @@ class QConv2d:
 
 
 __all__ = ["qconv_quantize_pack", "qconv_requant_params", "qconv_prepare_weights",
+           "qconv_s2d_desc", "qconv_quantize_pack_s2d", "qconv_prepare_weights_s2d",
            "qconv_prepared_weight_bytes", "qconv2d_workspace_size", "qconv2d_forward",
            "qconv_debug_im2col_tile", "make_desc", "qconv_desc", "QConv2d", "QConvError",
            "QC_U4", "QC_S4", "QC_U8", "QC_S8", "QC_S32", "out_hw", "lib_path"]

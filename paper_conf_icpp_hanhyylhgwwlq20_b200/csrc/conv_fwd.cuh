@@ -45,6 +45,11 @@ struct ConvParams {
     int32_t stride_h, stride_w, pad_h, pad_w, dil_h, dil_w;
     int32_t H, W, R, C8;              // C8 = channels (int8 bytes per pixel after widening)
     int32_t BK, bkp, stages, sw_layout, sw_mask;
+    int32_t pair;                     // C8 == 16: one K-stage = 2 filter taps x 16 B, no swizzle
+    int32_t y_tma;                    // epilogue stages the whole output tile in smem -> TMA store
+    uint32_t off_ystg;                // staging: n_ygroups x [128 rows x y_gw bytes], swizzled
+    int32_t y_gw, y_gmask, n_ygroups; // staging group width (32/64/128 B), swizzle mask, count
+    int32_t cvt_shift;                // log2(16-byte packed chunks per pixel) for the converter
     uint32_t idesc, tmem_cols;
     // shared memory carve-up (byte offsets from the 1024-aligned base)
     uint32_t off_a, off_b, off_stg, off_bar, off_par;
@@ -64,6 +69,11 @@ struct ConvParams {
 //       v = acc + b (int32, exact by the API contract)
 //       y = clamp((mulhi(v, m) + rhi) >> sh),  rhi = 2^(n-33) + zy*2^(n-32), sh = n-32
 //     exact: v*m + 2^(n-1) + zy*2^n = v*m + rhi*2^32, so floor(./2^n) = (floor(v*m/2^32)+rhi)>>sh
+//   mid chunk   {b, m, k, vlim}: 14 <= shift <= 33 for all 32 columns (k = 33-n, vlim = 2^(n-20)):
+//       x = clamp(acc + b, -vlim, vlim) << k;  y = clamp((mulhi(x, m) + 1 + 2zy) >> 1)
+//     exact: scaling numerator and denominator by 2^k gives shift 33; |acc+b| > 2^(n-20)
+//     already saturates every 8-bit output range (|t| >= 2^10), so the pre-clamp changes
+//     nothing and keeps x << k inside int32
 //   general chunk {b, m, n, 0}: t = (int64(v)*m + 2^(n-1)) >> n (int64), clamp, + zy
 //   S32 output   {b, 0, 0, 0}:  y = acc + b
 struct __align__(16) EpiCol {
@@ -102,6 +112,19 @@ __device__ __forceinline__ void epi_fast16(uint32_t (&v)[32], uint32_t par_addr,
         const int4 pr = lds128(par_addr + 16u * j);
         const int32_t x = static_cast<int32_t>(v[j]) + pr.x;
         const int32_t t = (__mulhi(x, pr.y) + pr.z) >> pr.w;
+        v[j] = static_cast<uint32_t>(min(hi, max(lo, t)));
+    }
+}
+
+template <int H>
+__device__ __forceinline__ void epi_mid16(uint32_t (&v)[32], uint32_t par_addr, int32_t lo,
+                                          int32_t hi, int32_t rmid) {
+#pragma unroll
+    for (int j = H; j < H + 16; ++j) {
+        const int4 pr = lds128(par_addr + 16u * j);
+        int32_t x = static_cast<int32_t>(v[j]) + pr.x;
+        x = min(pr.w, max(-pr.w, x)) << pr.z;
+        const int32_t t = (__mulhi(x, pr.y) + rmid) >> 1;
         v[j] = static_cast<uint32_t>(min(hi, max(lo, t)));
     }
 }
@@ -198,11 +221,56 @@ __device__ __forceinline__ void store16(const ConvParams &p, const uint32_t (&v)
     }
 }
 
+// Pack outputs v[H .. H+16) (output channels col .. col+16 of the tile) of row `row` into the
+// tile staging buffer: groups of y_gw bytes per row, each group a [128][y_gw] block with the
+// TMA swizzle of that width (16-byte unit index XOR address bits 7.., as the TMA store reads it).
+template <int OUT, int H>
+__device__ __forceinline__ void stage16(const ConvParams &p, const uint32_t (&v)[32], uint32_t sbase,
+                                        int row, int col) {
+    constexpr bool kInt4 = (OUT == OUT_U4 || OUT == OUT_S4);
+    const uint32_t ob = kInt4 ? static_cast<uint32_t>(col) / 2u : static_cast<uint32_t>(col);
+    const uint32_t gw = static_cast<uint32_t>(p.y_gw);
+    const uint32_t g = ob / gw, o = ob - g * gw;
+    const uint32_t off = static_cast<uint32_t>(row) * gw + o;
+    const uint32_t addr = sbase + g * 128u * gw + (off ^ (((off >> 7) & static_cast<uint32_t>(p.y_gmask)) << 4));
+    if (!kInt4) {
+        uint32_t w[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int32_t *y = reinterpret_cast<const int32_t *>(&v[H + 4 * j]);
+            if (OUT == OUT_U8)
+                w[j] = pack_sat_u8(y[1], y[0], pack_sat_u8(y[3], y[2], 0u));
+            else
+                w[j] = pack_sat_s8(y[1], y[0], pack_sat_s8(y[3], y[2], 0u));
+        }
+        sts128(addr, w[0], w[1], w[2], w[3]);
+    } else {
+        uint32_t w[2];
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+            const int32_t *y = reinterpret_cast<const int32_t *>(&v[H + 8 * j]);
+            if (OUT == OUT_U4) {
+                uint32_t t = pack_sat_u4(y[7], y[6], 0u);
+                t = pack_sat_u4(y[5], y[4], t);
+                t = pack_sat_u4(y[3], y[2], t);
+                w[j] = pack_sat_u4(y[1], y[0], t);
+            } else {
+                uint32_t t = pack_sat_s4(y[7], y[6], 0u);
+                t = pack_sat_s4(y[5], y[4], t);
+                t = pack_sat_s4(y[3], y[2], t);
+                w[j] = pack_sat_s4(y[1], y[0], t);
+            }
+        }
+        sts64(addr, w[0], w[1]);
+    }
+}
+
 template <int OUT, bool ZX, int H>
 __device__ __forceinline__ void epi_half(const ConvParams &p, uint32_t (&v)[32], uint32_t pa,
-                                         bool fast, int kc, int64_t m, bool row_ok, int zr0,
-                                         int zr1, int zs0, int zs1) {
-    if (fast) epi_fast16<H>(v, pa, p.clamp_lo, p.clamp_hi);
+                                         int mode, int32_t rmid, int kc, int64_t m, bool row_ok,
+                                         int zr0, int zr1, int zs0, int zs1) {
+    if (mode == 0) epi_fast16<H>(v, pa, p.clamp_lo, p.clamp_hi);
+    else if (mode == 1) epi_mid16<H>(v, pa, p.clamp_lo, p.clamp_hi, rmid);
     else epi_general16<OUT, ZX, H>(p, v, pa, kc - H, zr0, zr1, zs0, zs1);
     if (row_ok) store16<OUT, H>(p, v, kc, m);
 }
@@ -211,7 +279,7 @@ __device__ __forceinline__ void epi_half(const ConvParams &p, uint32_t (&v)[32],
 template <bool IS4, int OUT, bool ZX>
 __global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
 qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap wmap,
-                 const __grid_constant__ ConvParams p) {
+                 const __grid_constant__ CUtensorMap ymap, const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                                 ~uintptr_t(1023));
@@ -232,6 +300,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
     if (warp == kWarpTMA && lane == 0) {
         tma_prefetch_desc(&xmap);
         tma_prefetch_desc(&wmap);
+        if (p.y_tma) tma_prefetch_desc(&ymap);
         for (int i = 0; i < NS; ++i) {
             mbar_init(&full[i], 1);
             mbar_init(&empty[i], 1);
@@ -255,7 +324,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
         if (lane == 0) {
             int stage = 0;
             uint32_t phase = 0;
-            const uint32_t tx = static_cast<uint32_t>(kBM * p.bkp + p.BN * p.BK);
+            const uint32_t tx = static_cast<uint32_t>(kBM * (p.pair ? 32 : p.bkp) + p.BN * p.BK);
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
                 const int m0 = (tile / p.n_tiles_n) * kBM;
                 const int n0 = (tile % p.n_tiles_n) * p.BN;
@@ -265,6 +334,27 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 const int q0 = rem - p0 * p.Q;
                 const int wb = q0 * p.stride_w - p.pad_w;
                 const int hb = p0 * p.stride_h - p.pad_h;
+                if (p.pair) {
+                    const int RS = p.R * p.S;
+                    for (int kb = 0; kb < p.num_kb; ++kb) {
+                        const int t0 = 2 * kb, t1 = t0 + 1;
+                        const int r0 = t0 / p.S, s0 = t0 - r0 * p.S;
+                        int r1 = r0, s1 = s0, kg1 = RS * 16;        // odd tail: B slot OOB -> 0
+                        if (t1 < RS) { r1 = t1 / p.S; s1 = t1 - r1 * p.S; kg1 = t1 * 16; }
+                        mbar_wait(&empty[stage], phase ^ 1u);
+                        mbar_arrive_expect_tx(&full[stage], tx);
+                        uint8_t *adst = smem + p.off_a + stage * p.a_stage_bytes;
+                        uint8_t *bdst = smem + p.off_b + stage * p.b_stage_bytes;
+                        tma_load_im2col_4d(adst, &xmap, &full[stage], 0, wb, hb, img,
+                                           static_cast<uint16_t>(s0 * p.dil_w), static_cast<uint16_t>(r0 * p.dil_h));
+                        tma_load_im2col_4d(adst + kBM * 16, &xmap, &full[stage], 0, wb, hb, img,
+                                           static_cast<uint16_t>(s1 * p.dil_w), static_cast<uint16_t>(r1 * p.dil_h));
+                        tma_load_2d(bdst, &wmap, &full[stage], t0 * 16, n0);
+                        tma_load_2d(bdst + p.BN * 16, &wmap, &full[stage], kg1, n0);
+                        if (++stage == NS) { stage = 0; phase ^= 1u; }
+                    }
+                    continue;
+                }
                 for (int kb = 0; kb < p.num_kb; ++kb) {
                     const int r = kb / taps_per_r;
                     const int rem2 = kb - r * taps_per_r;
@@ -302,10 +392,18 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                     tc_fence_after();
                     const uint32_t a_addr = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
                     const uint32_t b_addr = smem_u32(smem + p.off_b + stage * p.b_stage_bytes);
-                    for (int k = 0; k < ksteps; ++k) {
-                        const uint64_t ad = make_smem_desc(a_addr + 32u * k, 16u, sbo, p.sw_layout);
-                        const uint64_t bd = make_smem_desc(b_addr + 32u * k, 16u, sbo, p.sw_layout);
-                        mma_i8(d_tmem, ad, bd, p.idesc, (kb | k) != 0 ? 1u : 0u);
+                    if (p.pair) {
+                        // canonical no-swizzle K-major: core matrices 8 rows x 16 B; the two
+                        // 16-byte K halves (filter taps) are LBO apart, 8-row groups SBO = 128 B
+                        const uint64_t ad = make_smem_desc(a_addr, kBM * 16u, 128u, 0u);
+                        const uint64_t bd = make_smem_desc(b_addr, static_cast<uint32_t>(p.BN) * 16u, 128u, 0u);
+                        mma_i8(d_tmem, ad, bd, p.idesc, kb != 0 ? 1u : 0u);
+                    } else {
+                        for (int k = 0; k < ksteps; ++k) {
+                            const uint64_t ad = make_smem_desc(a_addr + 32u * k, 16u, sbo, p.sw_layout);
+                            const uint64_t bd = make_smem_desc(b_addr + 32u * k, 16u, sbo, p.sw_layout);
+                            mma_i8(d_tmem, ad, bd, p.idesc, (kb | k) != 0 ? 1u : 0u);
+                        }
                     }
                     mma_commit(&empty[stage]);
                     if (++stage == NS) { stage = 0; phase ^= 1u; }
@@ -322,8 +420,10 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
         const uint32_t par_base = smem_u32(par);
         const int nchunks = (p.BN + 31) / 32;
         const bool force_general = (OUT == OUT_S32) || ZX;
+        const int32_t rmid = 1 + 2 * p.y_zero;
         int cached_n0 = -1;
         int it = 0;
+        const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
@@ -342,18 +442,23 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                     e.m = __ldg(p.mult + k);
                     nn = __ldg(p.shift + k);
                 }
-                const bool fast = !force_general &&
-                                  __ballot_sync(0xffffffffu, nn >= 33 && nn <= 52) == 0xffffffffu;
+                const bool all_fast = __ballot_sync(0xffffffffu, nn >= 33 && nn <= 52) == 0xffffffffu;
+                const bool all_mid =
+                    __ballot_sync(0xffffffffu, (nn >= 14 && nn <= 33) || k >= p.K) == 0xffffffffu;
+                const int mode = force_general ? 2 : (all_fast ? 0 : (all_mid ? 1 : 2));
                 if (OUT != OUT_S32 && k < p.K) {
-                    if (fast) {
+                    if (mode == 0) {
                         e.c2 = (1 << (nn - 33)) + p.y_zero * (1 << (nn - 32));
                         e.c3 = nn - 32;
+                    } else if (mode == 1) {
+                        e.c2 = 33 - nn;
+                        e.c3 = 1 << (nn - 20 > 0 ? nn - 20 : 0);
                     } else {
                         e.c2 = nn;
                     }
                 }
                 if (c < p.BN) *reinterpret_cast<EpiCol *>(reinterpret_cast<uint8_t *>(par) + 16 * c) = e;
-                if (lane == 0) chunk_fast[ew] = fast ? 1 : 0;
+                if (lane == 0) chunk_fast[ew] = static_cast<uint8_t>(mode);
                 named_bar_sync(1, kNumEpiWarps * 32);
                 cached_n0 = n0;
             }
@@ -373,46 +478,90 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
             const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
                                    static_cast<uint32_t>(buf * p.BN);
             uint32_t v[32];
-            for (int ci = half; ci < nchunks; ci += 2) {
-                const int col0 = ci * 32;
-                const int nc = min(32, p.BN - col0);
+            if (OUT != OUT_S32 && p.y_tma) {
+                // whole-tile staging in smem, written back by TMA stores of [128 rows x y_gw]
+                // groups (full 32..128-byte rows; rows >= M and columns >= K clipped by the map)
+                const bool storer = ew == 0 && lane == 0;
+                if (storer) bulk_wait_read<0>();          // previous tile's store has read staging
+                named_bar_sync(1, kNumEpiWarps * 32);
+                for (int ci = half; ci < nchunks; ci += 2) {
+                    const int col0 = ci * 32;
+                    __syncwarp();
+                    tmem_ld_32x32b_x32(taddr + col0, v);
+                    tmem_wait_ld();
+                    const uint32_t pa = par_base + 16u * col0;
+                    const int mode = chunk_fast[ci];
+                    if (mode == 0) {
+                        epi_fast16<0>(v, pa, p.clamp_lo, p.clamp_hi);
+                        epi_fast16<16>(v, pa, p.clamp_lo, p.clamp_hi);
+                    } else if (mode == 1) {
+                        epi_mid16<0>(v, pa, p.clamp_lo, p.clamp_hi, rmid);
+                        epi_mid16<16>(v, pa, p.clamp_lo, p.clamp_hi, rmid);
+                    } else {
+                        epi_general16<OUT, ZX, 0>(p, v, pa, n0 + col0, zr0, zr1, zs0, zs1);
+                        epi_general16<OUT, ZX, 16>(p, v, pa, n0 + col0, zr0, zr1, zs0, zs1);
+                    }
+                    stage16<OUT, 0>(p, v, ystg_base, row, col0);
+                    stage16<OUT, 16>(p, v, ystg_base, row, col0 + 16);
+                }
+                tc_fence_before();
                 __syncwarp();
-                if (nc == 32) tmem_ld_32x32b_x32(taddr + col0, v);
-                else tmem_ld_32x32b_x16(taddr + col0, v);
-                tmem_wait_ld();
-                const uint32_t pa = par_base + 16u * col0;
-                const bool fast = !force_general && chunk_fast[ci];
-                epi_half<OUT, ZX, 0>(p, v, pa, fast, n0 + col0, m, row_ok, zr0, zr1, zs0, zs1);
-                if (nc == 32)
-                    epi_half<OUT, ZX, 16>(p, v, pa, fast, n0 + col0 + 16, m, row_ok, zr0, zr1, zs0, zs1);
+                if (lane == 0) mbar_arrive(&tempty[buf]);    // accumulator drained: MMA may reuse it
+                fence_proxy_async_smem();
+                named_bar_sync(1, kNumEpiWarps * 32);
+                if (storer) {
+                    constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
+                    for (int g = 0; g < p.n_ygroups; ++g)
+                        tma_store_2d(&ymap, smem + p.off_ystg + g * 128 * p.y_gw,
+                                     n0 * kBits / 8 + g * p.y_gw, m0);
+                    bulk_commit();
+                }
+                continue;
+            } else {
+                for (int ci = half; ci < nchunks; ci += 2) {
+                    const int col0 = ci * 32;
+                    const int nc = min(32, p.BN - col0);
+                    __syncwarp();
+                    if (nc == 32) tmem_ld_32x32b_x32(taddr + col0, v);
+                    else tmem_ld_32x32b_x16(taddr + col0, v);
+                    tmem_wait_ld();
+                    const uint32_t pa = par_base + 16u * col0;
+                    const int mode = chunk_fast[ci];
+                    epi_half<OUT, ZX, 0>(p, v, pa, mode, rmid, n0 + col0, m, row_ok, zr0, zr1, zs0, zs1);
+                    if (nc == 32)
+                        epi_half<OUT, ZX, 16>(p, v, pa, mode, rmid, n0 + col0 + 16, m, row_ok, zr0, zr1, zs0, zs1);
+                }
             }
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&tempty[buf]);
         }
+        if (OUT != OUT_S32 && p.y_tma && ew == 0 && lane == 0) bulk_wait<0>();
     } else if (IS4 && warp >= kWarpCvt0 && warp < kWarpCvt0 + kNumCvtWarps) {
         // ===================== int4 -> int8 widening (4 warps) =====================
         const int ct = (warp - kWarpCvt0) * 32 + lane;      // 0..127
-        const int chunks_per_row = p.bkp / 16;               // 16-byte packed chunks per pixel
-        const int nchunks = kBM * chunks_per_row;
+        const int cshift = p.cvt_shift;                      // log2(16-byte packed chunks/pixel)
+        const int nchunks = kBM << cshift;
         const bool sgn = ((p.idesc >> 7) & 1u) != 0;
+        const uint32_t sw = static_cast<uint32_t>(p.sw_mask);
+        const uint32_t bkb = static_cast<uint32_t>(p.BK);
         int stage = 0;
         uint32_t phase = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
             for (int kb = 0; kb < p.num_kb; ++kb) {
                 mbar_wait(&full[stage], phase);
-                const uint8_t *stg = smem + p.off_stg + stage * p.stg_stage_bytes;
-                uint8_t *adst = smem + p.off_a + stage * p.a_stage_bytes;
+                const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
+                const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
                 for (int g = ct; g < nchunks; g += kNumCvtWarps * 32) {
-                    const int rr = g / chunks_per_row;
-                    const int cir = g - rr * chunks_per_row;
-                    const uint4 pk = *reinterpret_cast<const uint4 *>(stg + 16 * g);
-                    const uint32_t src[4] = {pk.x, pk.y, pk.z, pk.w};
+                    const uint32_t rr = static_cast<uint32_t>(g) >> cshift;
+                    const uint32_t cir = static_cast<uint32_t>(g) & ((1u << cshift) - 1u);
+                    const uint4 pk = lds128u(stg + 16u * static_cast<uint32_t>(g));
+                    const uint32_t src4[4] = {pk.x, pk.y, pk.z, pk.w};
                     uint32_t o[8];
 #pragma unroll
                     for (int j = 0; j < 4; ++j) {
-                        uint32_t lo = src[j] & 0x0F0F0F0Fu;
-                        uint32_t hi = (src[j] >> 4) & 0x0F0F0F0Fu;
+                        uint32_t lo = src4[j] & 0x0F0F0F0Fu;
+                        uint32_t hi = (src4[j] >> 4) & 0x0F0F0F0Fu;
                         if (sgn) {
                             lo = ((lo ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
                             hi = ((hi ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
@@ -421,13 +570,10 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                         o[2 * j + 1] = __byte_perm(lo, hi, 0x7362);
                     }
                     // widened bytes [32*cir, 32*cir+32) of row rr, swizzled like the TMA would
-                    const uint32_t off0 = static_cast<uint32_t>(rr * p.BK + 32 * cir);
+                    const uint32_t off0 = rr * bkb + 32u * cir;
                     const uint32_t off1 = off0 + 16u;
-                    const uint32_t sw = static_cast<uint32_t>(p.sw_mask);
-                    const uint32_t ph0 = off0 ^ (((off0 >> 7) & sw) << 4);
-                    const uint32_t ph1 = off1 ^ (((off1 >> 7) & sw) << 4);
-                    *reinterpret_cast<uint4 *>(adst + ph0) = make_uint4(o[0], o[1], o[2], o[3]);
-                    *reinterpret_cast<uint4 *>(adst + ph1) = make_uint4(o[4], o[5], o[6], o[7]);
+                    sts128(adst + (off0 ^ (((off0 >> 7) & sw) << 4)), o[0], o[1], o[2], o[3]);
+                    sts128(adst + (off1 ^ (((off1 >> 7) & sw) << 4)), o[4], o[5], o[6], o[7]);
                 }
                 fence_proxy_async_smem();
                 __syncwarp();

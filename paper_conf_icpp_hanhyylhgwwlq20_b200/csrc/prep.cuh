@@ -161,4 +161,81 @@ __global__ void zx_table_kernel(const int8_t *__restrict__ w8, int32_t *__restri
     }
 }
 
+// ---------------------------------------------------------------------------
+// Space-to-depth (2x2) form of a stride-2 convolution (the C=3 stem).
+// X2[n,i,j,(2b+b')*c+cc] = q(x[n, 2i+b-pad_h, 2j+b'-pad_w, cc]) (code z outside the image
+// or beyond 4c), one code per byte, so that a 7x7/s2 conv over C=3 becomes a 4x4/s1 conv over
+// C2=16 with W2[k,a,a',(2b+b')*c+cc] = w[k, 2a+b, 2a'+b', cc] (0 beyond R, S): the same sums.
+struct QuantS2DParams {
+    const void *x;
+    uint8_t *y;
+    int32_t n, h, w, c, hs, ws, cs, pad_h, pad_w;
+    float inv_s, flo, fhi;
+    int32_t z, qmin, qmax, bf16;
+};
+
+__global__ void __launch_bounds__(256) quantize_s2d_kernel(const __grid_constant__ QuantS2DParams p) {
+    QuantParams qp;
+    qp.x = p.x; qp.inv_s = p.inv_s; qp.flo = p.flo; qp.fhi = p.fhi;
+    qp.z = p.z; qp.qmin = p.qmin; qp.qmax = p.qmax; qp.bf16 = p.bf16;
+    const int64_t total = static_cast<int64_t>(p.n) * p.hs * p.ws;
+    const int32_t c4 = 4 * p.c;
+    for (int64_t t = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; t < total;
+         t += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t img = t / (static_cast<int64_t>(p.hs) * p.ws);
+        const int32_t rem = static_cast<int32_t>(t - img * p.hs * p.ws);
+        const int32_t i = rem / p.ws, j = rem - (rem / p.ws) * p.ws;
+        uint8_t *dst = p.y + t * p.cs;
+        for (int32_t ch0 = 0; ch0 < p.cs; ch0 += 16) {
+            uint32_t w[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+            for (int jj = 0; jj < 16; ++jj) {
+                const int32_t ch = ch0 + jj;
+                int32_t code = p.z;
+                if (ch < c4) {
+                    const int32_t blk = ch / p.c, cc = ch - blk * p.c;
+                    const int32_t hh = 2 * i + (blk >> 1) - p.pad_h;
+                    const int32_t ww = 2 * j + (blk & 1) - p.pad_w;
+                    if (hh >= 0 && hh < p.h && ww >= 0 && ww < p.w)
+                        code = quantize_one(load_x(qp, ((img * p.h + hh) * p.w + ww) * p.c + cc), qp);
+                }
+                w[jj >> 2] |= static_cast<uint32_t>(code & 0xFF) << (8 * (jj & 3));
+            }
+            *reinterpret_cast<uint4 *>(dst + ch0) = make_uint4(w[0], w[1], w[2], w[3]);
+        }
+    }
+}
+
+// W2 (int8 KRSC of the transformed conv) from packed w (4- or 8-bit codes).
+__global__ void __launch_bounds__(256) weights_s2d_kernel(const uint8_t *__restrict__ w,
+                                                          int8_t *__restrict__ w2, int32_t k, int32_t r,
+                                                          int32_t s, int32_t c, int32_t r2, int32_t s2,
+                                                          int32_t cs, int32_t bits, int32_t is_signed) {
+    const int64_t total = static_cast<int64_t>(k) * r2 * s2 * cs;
+    for (int64_t e = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; e < total;
+         e += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        int64_t rest = e;
+        const int32_t ch = static_cast<int32_t>(rest % cs); rest /= cs;
+        const int32_t a2 = static_cast<int32_t>(rest % s2); rest /= s2;
+        const int32_t a1 = static_cast<int32_t>(rest % r2); rest /= r2;
+        const int32_t kk = static_cast<int32_t>(rest);
+        int32_t v = 0;
+        if (ch < 4 * c) {
+            const int32_t blk = ch / c, cc = ch - blk * c;
+            const int32_t rr = 2 * a1 + (blk >> 1), ss = 2 * a2 + (blk & 1);
+            if (rr < r && ss < s) {
+                const int64_t idx = ((static_cast<int64_t>(kk) * r + rr) * s + ss) * c + cc;
+                if (bits == 8) {
+                    v = is_signed ? static_cast<int32_t>(static_cast<int8_t>(w[idx])) : static_cast<int32_t>(w[idx]);
+                } else {
+                    const uint8_t b = w[idx >> 1];
+                    v = (idx & 1) ? (b >> 4) : (b & 0xF);
+                    if (is_signed && v >= 8) v -= 16;
+                }
+            }
+        }
+        w2[e] = static_cast<int8_t>(v);
+    }
+}
+
 }  // namespace qc

@@ -160,7 +160,8 @@ qc_status validate_desc(const qconv_desc *d, Geometry *g) {
 // Support + overflow checks for the GPU path (after validate_desc).
 qc_status check_supported(const qconv_desc *d, const Geometry &g) {
     if (dtype_bits(d->x_t) != dtype_bits(d->w_t)) return QC_ERR_UNSUPPORTED;   // mixed widths: NEXT
-    if (d->c % 32) return QC_ERR_UNSUPPORTED;          // MMA K granularity / 16-byte TMA strides
+    const bool pair = dtype_bits(d->x_t) == 8 && d->c == 16;   // 2 taps per 32-byte K-stage
+    if (d->c % 32 && !pair) return QC_ERR_UNSUPPORTED;   // MMA K granularity / 16-byte TMA strides
     if (d->stride_h > 8 || d->stride_w > 8) return QC_ERR_UNSUPPORTED;   // TMA traversal stride
     const int lw = -d->pad_w, lh = -d->pad_h;
     const int uw = d->pad_w - d->dil_w * (d->s - 1), uh = d->pad_h - d->dil_h * (d->r - 1);
@@ -197,10 +198,11 @@ uint32_t pow2_cols(int n) {
 
 qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const bool is4 = g.bits == 4;
-    pl->BK = choose_bk(d->c);
-    pl->bkp = is4 ? pl->BK / 2 : pl->BK;
-    pl->chunks = d->c / pl->BK;
-    pl->num_kb = d->r * d->s * pl->chunks;
+    const bool pair = !is4 && d->c == 16;
+    pl->BK = pair ? 32 : choose_bk(d->c);
+    pl->bkp = is4 ? pl->BK / 2 : (pair ? 16 : pl->BK);
+    pl->chunks = pair ? 1 : d->c / pl->BK;
+    pl->num_kb = pair ? (d->r * d->s + 1) / 2 : d->r * d->s * pl->chunks;
     const int m_tiles = static_cast<int>((g.M + qc::kBM - 1) / qc::kBM);
     const int sms = num_sms();
     int BN = std::min(qc::kMaxBN, ((d->k + 15) / 16) * 16);
@@ -217,7 +219,14 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const uint32_t b_bytes = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * pl->BK, 1024));
     const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(qc::kBM * pl->bkp) : 0u;
     const uint32_t per_stage = a_bytes + b_bytes + stg_bytes;
-    const uint32_t fixed = static_cast<uint32_t>(qc::kMaxBN) * 16u + 64u + 1024u;  // params, flags, barriers
+    const int ybits = dtype_bits(d->y_t);
+    const int tile_row_bytes = BN * ybits / 8;
+    const int y_gw = tile_row_bytes >= 128 ? 128 : tile_row_bytes;
+    const bool y_tma = d->y_t != QC_S32 && BN % 32 == 0 &&
+                       (static_cast<int64_t>(d->k) * ybits / 8) % 16 == 0 &&
+                       (y_gw == 32 || y_gw == 64 || (y_gw == 128 && tile_row_bytes % 128 == 0));
+    const uint32_t ystg_bytes = y_tma ? 128u * static_cast<uint32_t>(tile_row_bytes) : 0u;
+    const uint32_t fixed = static_cast<uint32_t>(qc::kMaxBN) * 16u + 64u + 1024u + ystg_bytes;
     const uint32_t budget = 227u * 1024u - 1024u - fixed;
     int stages = static_cast<int>(budget / per_stage);
     stages = std::min(stages, 8);
@@ -228,7 +237,12 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.off_a = 0;
     p.off_b = p.off_a + a_bytes * stages;
     p.off_stg = p.off_b + b_bytes * stages;
-    p.off_par = static_cast<uint32_t>(align_up(p.off_stg + stg_bytes * stages, 16));
+    p.off_ystg = static_cast<uint32_t>(align_up(p.off_stg + stg_bytes * stages, 1024));
+    p.y_tma = y_tma ? 1 : 0;
+    p.y_gw = y_gw;
+    p.y_gmask = y_gw == 128 ? 7 : (y_gw == 64 ? 3 : 1);
+    p.n_ygroups = y_tma ? tile_row_bytes / y_gw : 0;
+    p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + ystg_bytes, 16));
     p.off_bar = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 64u, 8));
     const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 4) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;       // + alignment slack for the 1024-B base
@@ -262,6 +276,8 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.bkp = pl->bkp;
     p.stages = stages;
     p.sw_layout = pl->BK == 128 ? 2 : (pl->BK == 64 ? 4 : 6);
+    p.pair = pair ? 1 : 0;
+    p.cvt_shift = pl->bkp >= 64 ? 2 : (pl->bkp >= 32 ? 1 : 0);
     p.sw_mask = pl->BK == 128 ? 7 : (pl->BK == 64 ? 3 : 1);
     p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), dtype_signed(d->x_t), dtype_signed(d->w_t));
     p.tmem_cols = pl->tmem_cols;
@@ -299,7 +315,7 @@ qc_status encode_x_map(const qconv_desc *d, const Geometry &g, const void *x, in
 }
 
 qc_status encode_w_map(const qconv_desc *d, const Geometry &g, const void *w8, int bk, int bn,
-                       CUtensorMap *map) {
+                       CUtensorMapSwizzle sw, CUtensorMap *map) {
     const Driver &drv = driver();
     if (!drv.tiled) return cuda_fail(drv.err);
     const cuuint64_t kg = static_cast<cuuint64_t>(d->r) * d->s * d->c;
@@ -308,16 +324,33 @@ qc_status encode_w_map(const qconv_desc *d, const Geometry &g, const void *w8, i
     cuuint32_t box[2] = {static_cast<cuuint32_t>(bk), static_cast<cuuint32_t>(bn)};
     cuuint32_t estr[2] = {1, 1};
     CUresult r = drv.tiled(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<void *>(w8), dims,
-                           strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_for(bk),
+                           strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
     small_tensor_fixup(map, static_cast<uint64_t>(g.w8_bytes));
     return QC_OK;
 }
 
+qc_status encode_y_map(const qconv_desc *d, const Geometry &g, void *y, int gw, CUtensorMap *map) {
+    const Driver &drv = driver();
+    if (!drv.tiled) return cuda_fail(drv.err);
+    const int yb = dtype_bits(d->y_t);
+    const cuuint64_t row = static_cast<cuuint64_t>(d->k) * yb / 8;
+    cuuint64_t dims[2] = {row, static_cast<cuuint64_t>(g.M)};
+    cuuint64_t strides[1] = {row};
+    cuuint32_t box[2] = {static_cast<cuuint32_t>(gw), static_cast<cuuint32_t>(qc::kBM)};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = drv.tiled(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, y, dims, strides, box, estr,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_for(gw),
+                           CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+    small_tensor_fixup(map, static_cast<uint64_t>(g.y_bytes));
+    return QC_OK;
+}
+
 template <bool IS4, int OUT, bool ZX>
 qc_status launch_conv_t(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
-                        cudaStream_t stream) {
+                        const CUtensorMap &ym, cudaStream_t stream) {
     auto kern = qc::qconv_fwd_kernel<IS4, OUT, ZX>;
     static int configured_smem = 0;   // per instantiation; max over calls is safe to keep
     if (configured_smem < static_cast<int>(pl.smem_bytes)) {
@@ -334,16 +367,16 @@ qc_status launch_conv_t(const Plan &pl, const CUtensorMap &xm, const CUtensorMap
     cfg.stream = stream;
     cfg.attrs = nullptr;
     cfg.numAttrs = 0;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, pl.cp);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, pl.cp);
     if (e != cudaSuccess) return cuda_fail(e);
     return QC_OK;
 }
 
 template <bool IS4, int OUT>
 qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
-                      cudaStream_t stream) {
-    return pl.cp.x_zero != 0 ? launch_conv_t<IS4, OUT, true>(pl, xm, wm, stream)
-                             : launch_conv_t<IS4, OUT, false>(pl, xm, wm, stream);
+                      const CUtensorMap &ym, cudaStream_t stream) {
+    return pl.cp.x_zero != 0 ? launch_conv_t<IS4, OUT, true>(pl, xm, wm, ym, stream)
+                             : launch_conv_t<IS4, OUT, false>(pl, xm, wm, ym, stream);
 }
 
 }  // namespace
@@ -525,20 +558,119 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
     p.y = y;
 
     alignas(64) CUtensorMap xm, wm;
-    s = encode_x_map(d, g, x, pl.bkp, g.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(pl.BK), &xm);
+    const bool pair = p.pair != 0;
+    s = encode_x_map(d, g, x, pl.bkp,
+                     (g.bits == 4 || pair) ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(pl.BK), &xm);
     if (s != QC_OK) return s;
-    s = encode_w_map(d, g, w8, pl.BK, pl.BN, &wm);
+    s = encode_w_map(d, g, w8, pair ? 16 : pl.BK, pl.BN,
+                     pair ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(pl.BK), &wm);
     if (s != QC_OK) return s;
 
+    alignas(64) CUtensorMap ym;
+    std::memset(&ym, 0, sizeof(ym));
+    if (p.y_tma) {
+        s = encode_y_map(d, g, y, p.y_gw, &ym);
+        if (s != QC_OK) return s;
+    }
     const bool is4 = g.bits == 4;
     switch (d->y_t) {
-        case QC_S32: return is4 ? launch_conv<true, qc::OUT_S32>(pl, xm, wm, st) : launch_conv<false, qc::OUT_S32>(pl, xm, wm, st);
-        case QC_U8: return is4 ? launch_conv<true, qc::OUT_U8>(pl, xm, wm, st) : launch_conv<false, qc::OUT_U8>(pl, xm, wm, st);
-        case QC_S8: return is4 ? launch_conv<true, qc::OUT_S8>(pl, xm, wm, st) : launch_conv<false, qc::OUT_S8>(pl, xm, wm, st);
-        case QC_U4: return is4 ? launch_conv<true, qc::OUT_U4>(pl, xm, wm, st) : launch_conv<false, qc::OUT_U4>(pl, xm, wm, st);
-        case QC_S4: return is4 ? launch_conv<true, qc::OUT_S4>(pl, xm, wm, st) : launch_conv<false, qc::OUT_S4>(pl, xm, wm, st);
+        case QC_S32: return is4 ? launch_conv<true, qc::OUT_S32>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_S32>(pl, xm, wm, ym, st);
+        case QC_U8: return is4 ? launch_conv<true, qc::OUT_U8>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_U8>(pl, xm, wm, ym, st);
+        case QC_S8: return is4 ? launch_conv<true, qc::OUT_S8>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_S8>(pl, xm, wm, ym, st);
+        case QC_U4: return is4 ? launch_conv<true, qc::OUT_U4>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_U4>(pl, xm, wm, ym, st);
+        case QC_S4: return is4 ? launch_conv<true, qc::OUT_S4>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_S4>(pl, xm, wm, ym, st);
     }
     return QC_ERR_INVALID_ARG;
+}
+
+// ------------------------------------------------------------------ space-to-depth stem
+static int32_t s2d_channels(int32_t c) {
+    const int32_t c4 = 4 * c;
+    return c4 <= 16 ? 16 : (c4 + 31) / 32 * 32;
+}
+static qc_dtype byte_container(qc_dtype t) {
+    return (t == QC_U4 || t == QC_U8) ? QC_U8 : QC_S8;
+}
+
+qc_status qconv_s2d_desc(const qconv_desc *d, qconv_desc *out) {
+    if (!d) return QC_ERR_INVALID_ARG;
+    // the original activations are float (quantized by qconv_quantize_pack_s2d), so an odd c
+    // with a 4-bit code type is fine: validate the byte-container view
+    qconv_desc dv = *d;
+    dv.x_t = byte_container(d->x_t);
+    Geometry g;
+    qc_status s = validate_desc(&dv, &g);
+    if (s != QC_OK) return s;
+    if (!is_int_input(d->x_t) || d->x_zero < dtype_min(d->x_t) || d->x_zero > dtype_max(d->x_t))
+        return QC_ERR_INVALID_ARG;
+    if (!out) return QC_ERR_INVALID_ARG;
+    if (d->stride_h != 2 || d->stride_w != 2 || d->dil_h != 1 || d->dil_w != 1)
+        return QC_ERR_UNSUPPORTED;
+    qconv_desc o = *d;
+    o.r = (d->r + 1) / 2;
+    o.s = (d->s + 1) / 2;
+    o.h = g.P + o.r - 1;
+    o.w = g.Q + o.s - 1;
+    o.c = s2d_channels(d->c);
+    o.stride_h = o.stride_w = 1;
+    o.pad_h = o.pad_w = 0;
+    o.dil_h = o.dil_w = 1;
+    o.x_t = byte_container(d->x_t);
+    o.w_t = byte_container(d->w_t);
+    o.w_prepared = 1;
+    *out = o;
+    return QC_OK;
+}
+
+qc_status qconv_quantize_pack_s2d(const qconv_desc *d, const void *x, qc_ftype xt, float scale,
+                                  void *y, void *stream) {
+    qconv_desc o;
+    qc_status s = qconv_s2d_desc(d, &o);
+    if (s != QC_OK) return s;
+    if (!x || !y || (xt != QC_F32 && xt != QC_BF16)) return QC_ERR_INVALID_ARG;
+    if (!(scale > 0.0f) || !std::isfinite(scale)) return QC_ERR_INVALID_ARG;
+    if (!aligned16(x) || !aligned16(y)) return QC_ERR_MISALIGNED;
+    qc::QuantS2DParams p;
+    p.x = x;
+    p.y = static_cast<uint8_t *>(y);
+    p.n = d->n; p.h = d->h; p.w = d->w; p.c = d->c;
+    p.hs = o.h; p.ws = o.w; p.cs = o.c;
+    p.pad_h = d->pad_h; p.pad_w = d->pad_w;
+    p.inv_s = 1.0f / scale;
+    p.z = d->x_zero;
+    p.qmin = static_cast<int32_t>(dtype_min(d->x_t));
+    p.qmax = static_cast<int32_t>(dtype_max(d->x_t));
+    p.flo = static_cast<float>(p.qmin - p.z - 1);
+    p.fhi = static_cast<float>(p.qmax - p.z + 1);
+    p.bf16 = xt == QC_BF16;
+    const int64_t total = static_cast<int64_t>(p.n) * p.hs * p.ws;
+    const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, static_cast<int64_t>(num_sms()) * 16));
+    qc::quantize_s2d_kernel<<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(p);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e);
+    return QC_OK;
+}
+
+size_t qconv_prepared_weight_bytes_s2d(const qconv_desc *d) {
+    qconv_desc o;
+    if (qconv_s2d_desc(d, &o) != QC_OK) return 0;
+    return static_cast<size_t>(o.k) * o.r * o.s * o.c;
+}
+
+qc_status qconv_prepare_weights_s2d(const qconv_desc *d, const void *w, void *w_prep, void *stream) {
+    qconv_desc o;
+    qc_status s = qconv_s2d_desc(d, &o);
+    if (s != QC_OK) return s;
+    if (!w || !w_prep) return QC_ERR_INVALID_ARG;
+    if (!aligned16(w) || !aligned16(w_prep)) return QC_ERR_MISALIGNED;
+    const int64_t total = static_cast<int64_t>(o.k) * o.r * o.s * o.c;
+    const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, 4096));
+    qc::weights_s2d_kernel<<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(
+        static_cast<const uint8_t *>(w), static_cast<int8_t *>(w_prep), d->k, d->r, d->s, d->c, o.r,
+        o.s, o.c, dtype_bits(d->w_t), dtype_signed(d->w_t) ? 1 : 0);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e);
+    return QC_OK;
 }
 
 qc_status qconv_debug_im2col_tile(const qconv_desc *d, const void *x, int64_t m0, int32_t r,

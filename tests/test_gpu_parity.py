@@ -200,6 +200,21 @@ def test_conv_requant_shift_modes():
     np.testing.assert_array_equal(got, ref)
 
 
+@pytest.mark.parametrize("bits,lo_n,hi_n", [(8, 14, 33), (4, 14, 33), (8, 33, 52), (4, 28, 36)])
+def test_conv_requant_shift_ranges(bits, lo_n, hi_n):
+    """Random per-channel (m, shift) over whole 32-channel chunks: exercises the mid (shift
+    14..33, pre-clamped and rescaled), fast (33..52) and mixed/general epilogue branches,
+    including saturation, against the oracle's exact int128 rounding."""
+    cs = ConvShape("shr", 2, 9, 9, 64, 96, 3, 3, 1, 1)
+    li = make_layer_inputs(cs, bits, seed=lo_n * 7 + bits, relu=False, signed_out=True)
+    rng = np.random.default_rng(lo_n + hi_n)
+    m = rng.integers(1 << 30, 1 << 31, size=cs.k).astype(np.int32)
+    n = rng.integers(lo_n, hi_n + 1, size=cs.k).astype(np.int32)
+    ref = oracle.conv2d_layer(li, mult=m, shift=n)
+    got = _gpu_conv(li, m, n)
+    np.testing.assert_array_equal(got, ref)
+
+
 # ----------------------------------------------------------------------------- paper configs
 def test_config1_c1_8bit():
     """BASELINE configs[0]: 8-bit 3x3, N=1, C=K=64, 56x56, s1 p1, requantized int8 output."""
@@ -255,3 +270,47 @@ def test_vgg16_batch2_8bit():
         if cs.c == 3:
             continue
         _check_layer(make_layer_inputs(cs, 8, seed=3000 + i))
+
+
+# ----------------------------------------------------------------------------- C = 16 and the stem
+@pytest.mark.parametrize("cs", [ConvShape("p1", 2, 9, 11, 16, 48, 3, 3, 1, 1),
+                                ConvShape("p2", 1, 12, 12, 16, 64, 4, 4, 1, 0),
+                                ConvShape("p3", 3, 10, 7, 16, 16, 5, 5, 2, 2),
+                                ConvShape("p4", 1, 8, 8, 16, 32, 1, 1, 1, 0)], ids=lambda c: c.name)
+def test_conv_c16_tap_pairs(cs):
+    """8-bit C = 16: two filter taps per 32-byte K step (odd tap counts included)."""
+    _check_layer(make_layer_inputs(cs, 8, seed=41))
+    _check_layer(make_layer_inputs(cs, 8, seed=42, relu=False, signed_out=True))
+
+
+@pytest.mark.parametrize("bits", [8, 4])
+@pytest.mark.parametrize("n,x_zero", [(2, 0), (1, 3)])
+def test_stem_space_to_depth(bits, n, x_zero):
+    """7x7/s2/p3 C=3 stem through qconv_quantize_pack_s2d + prepare_weights_s2d + forward on
+    the transformed 4x4/s1 C=16 conv, against the oracle's direct 7x7 conv."""
+    from workloads import resnet50_convs
+    cs = resnet50_convs(n)[0]
+    rng = np.random.default_rng(100 + bits)
+    xf = float_image(rng, (n, cs.h, cs.w, cs.c))
+    xt = U4 if bits == 4 else U8
+    s_x = 3.0 / 15 if bits == 4 else 3.0 / 255
+    li = make_layer_inputs(cs, bits, seed=7 + bits, c_store=4)
+    li.x_zero = x_zero
+    xq = oracle.quantize(xf, s_x, x_zero, xt, c_pad=4)
+    li.x_bytes = xq
+    m, n_ = oracle.requant_params(li.s_x, li.s_w, li.s_y)
+    ref = oracle.conv2d_layer(li, mult=m, shift=n_)
+    d = qc.make_desc(n, cs.h, cs.w, 3, cs.k, 7, 7, stride=2, pad=3, x_t=xt, w_t=li.w_t,
+                     y_t=li.y_t, x_zero=x_zero, clamp_lo=li.clamp_lo, clamp_hi=li.clamp_hi)
+    w3 = pack_codes(li.w_codes[..., :3], li.w_t) if bits == 8 else None
+    if bits == 4:   # 4-bit rows of 3 channels are not byte aligned: pass 8-bit codes of s4 values
+        d.w_t = S8
+        w3 = pack_codes(li.w_codes[..., :3], S8)
+    d2 = qc.qconv_s2d_desc(d)
+    assert (d2.h, d2.w, d2.c, d2.r, d2.s) == (115, 115, 16, 4, 4)
+    x2 = qc.qconv_quantize_pack_s2d(d, torch.from_numpy(xf).to(DEV), s_x)
+    w2 = qc.qconv_prepare_weights_s2d(d, torch.from_numpy(np.ascontiguousarray(w3)).to(DEV))
+    y = qc.qconv2d_forward(d2, x2, w2, torch.from_numpy(li.bias).to(DEV),
+                           torch.from_numpy(m).to(DEV), torch.from_numpy(n_).to(DEV))
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(y.cpu().numpy(), ref)

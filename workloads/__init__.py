@@ -306,8 +306,9 @@ def make_layer_params(cs: ConvShape, bits: int, seed: int, *, c_store: Optional[
     s_x = np.float32(0.05)
     s_y = np.float32(float(s_x) * float(np.median(s_w)) * 2.33 * sigma_acc / DTYPE_RANGE[y_t][1])
     lo, hi = DTYPE_RANGE[y_t]
+    packable = DTYPE_BITS[w_t] == 8 or w_codes.shape[-1] % 2 == 0
     return LayerParams(shape=cs, x_t=x_t, w_t=w_t, y_t=y_t, w_codes=w_codes,
-                       w_bytes=pack_codes(w_codes, w_t), bias=bias, s_x=float(s_x), s_w=s_w,
+                       w_bytes=pack_codes(w_codes, w_t) if packable else None, bias=bias, s_x=float(s_x), s_w=s_w,
                        s_y=float(s_y), clamp_lo=max(lo, 0) if relu else lo, clamp_hi=hi,
                        c_store=c_st)
 
