@@ -31,6 +31,7 @@ constexpr int kBM = 128;             // output pixels per tile (UMMA M)
 constexpr int kMaxBN = 256;
 constexpr int kWarpTMA = 0;
 constexpr int kWarpMMA = 1;
+constexpr int kNumProducers = 3;      // TMA issuers: lane 0 of warps 0, 2, 3
 constexpr int kWarpEpi0 = 4;         // warps 4..11: epilogue (TMEM lane quarter = warp % 4)
 constexpr int kNumEpiWarps = 8;
 constexpr int kWarpCvt0 = 12;        // warps 12..15: int4 -> int8 converters (4-bit only)
@@ -50,6 +51,10 @@ struct ConvParams {
     uint32_t off_ystg;                // staging: n_ygroups x [128 rows x y_gw bytes], swizzled
     int32_t y_gw, y_gmask, n_ygroups; // staging group width (32/64/128 B), swizzle mask, count
     int32_t cvt_shift;                // log2(16-byte packed chunks per pixel) for the converter
+    int32_t need_clamp;               // clamp range narrower than the output dtype range
+    unsigned long long *trace;        // debug: per-event timestamps of CTA 0 (QC_TRACE), or null
+    int32_t exp_flags;                // debug experiments (QC_EXPERIMENT): 1 no B reload, 2 no A reload,
+                                      // 4 no MMA, 8 epilogue: TMEM loads only, 16 epilogue: nothing
     uint32_t idesc, tmem_cols;
     // shared memory carve-up (byte offsets from the 1024-aligned base)
     uint32_t off_a, off_b, off_stg, off_bar, off_par;
@@ -69,11 +74,12 @@ struct ConvParams {
 //       v = acc + b (int32, exact by the API contract)
 //       y = clamp((mulhi(v, m) + rhi) >> sh),  rhi = 2^(n-33) + zy*2^(n-32), sh = n-32
 //     exact: v*m + 2^(n-1) + zy*2^n = v*m + rhi*2^32, so floor(./2^n) = (floor(v*m/2^32)+rhi)>>sh
-//   mid chunk   {b, m, k, vlim}: 14 <= shift <= 33 for all 32 columns (k = 33-n, vlim = 2^(n-20)):
-//       x = clamp(acc + b, -vlim, vlim) << k;  y = clamp((mulhi(x, m) + 1 + 2zy) >> 1)
-//     exact: scaling numerator and denominator by 2^k gives shift 33; |acc+b| > 2^(n-20)
-//     already saturates every 8-bit output range (|t| >= 2^10), so the pre-clamp changes
-//     nothing and keeps x << k inside int32
+//   mid chunk   {b, m, k, vlim}: 20 <= shift <= 50 for all 32 columns; T = max(33, max shift
+//     of the chunk), k = T-n, vlim = 2^(n-20); per chunk rhiT = 2^(T-33) + zy*2^(T-32):
+//       x = clamp(acc + b, -vlim, vlim) << k;  y = clamp((mulhi(x, m) + rhiT) >> (T-32))
+//     exact: scaling numerator and denominator by 2^k gives the common shift T; |acc+b| >
+//     2^(n-20) already saturates every 8-bit output range (|t| >= 2^10), so the pre-clamp
+//     changes nothing and keeps |x << k| <= 2^30
 //   general chunk {b, m, n, 0}: t = (int64(v)*m + 2^(n-1)) >> n (int64), clamp, + zy
 //   S32 output   {b, 0, 0, 0}:  y = acc + b
 struct __align__(16) EpiCol {
@@ -103,8 +109,13 @@ __device__ __forceinline__ void valid_tap_range(int o, int stride, int pad, int 
     t1 = max(lo, hi);
 }
 
+template <int OUT, bool ZX, int H>
+__device__ __forceinline__ void epi_general16(const ConvParams &p, uint32_t (&v)[32],
+                                              uint32_t par_addr, int kc, int zr0, int zr1,
+                                              int zs0, int zs1);
+
 // Fast chunk: 32 columns, all constants from smem (broadcast LDS.128), no branches.
-template <int H>
+template <int H, bool CLAMP>
 __device__ __forceinline__ void epi_fast16(uint32_t (&v)[32], uint32_t par_addr, int32_t lo,
                                            int32_t hi) {
 #pragma unroll
@@ -112,20 +123,35 @@ __device__ __forceinline__ void epi_fast16(uint32_t (&v)[32], uint32_t par_addr,
         const int4 pr = lds128(par_addr + 16u * j);
         const int32_t x = static_cast<int32_t>(v[j]) + pr.x;
         const int32_t t = (__mulhi(x, pr.y) + pr.z) >> pr.w;
-        v[j] = static_cast<uint32_t>(min(hi, max(lo, t)));
+        v[j] = static_cast<uint32_t>(CLAMP ? min(hi, max(lo, t)) : t);
     }
 }
 
-template <int H>
+template <int H, bool CLAMP>
 __device__ __forceinline__ void epi_mid16(uint32_t (&v)[32], uint32_t par_addr, int32_t lo,
-                                          int32_t hi, int32_t rmid) {
+                                          int32_t hi, int32_t rhi, int32_t sh) {
 #pragma unroll
     for (int j = H; j < H + 16; ++j) {
         const int4 pr = lds128(par_addr + 16u * j);
         int32_t x = static_cast<int32_t>(v[j]) + pr.x;
         x = min(pr.w, max(-pr.w, x)) << pr.z;
-        const int32_t t = (__mulhi(x, pr.y) + rmid) >> 1;
-        v[j] = static_cast<uint32_t>(min(hi, max(lo, t)));
+        const int32_t t = (__mulhi(x, pr.y) + rhi) >> sh;
+        v[j] = static_cast<uint32_t>(CLAMP ? min(hi, max(lo, t)) : t);
+    }
+}
+
+// Requantize the 32 accumulators of one chunk in place (mode per chunk, see EpiCol).
+template <int OUT, bool ZX, int H>
+__device__ __forceinline__ void epi_requant16(const ConvParams &p, uint32_t (&v)[32], uint32_t pa,
+                                              int4 ci, int kc, int zr0, int zr1, int zs0, int zs1) {
+    if (ci.x == 0) {
+        if (p.need_clamp) epi_fast16<H, true>(v, pa, p.clamp_lo, p.clamp_hi);
+        else epi_fast16<H, false>(v, pa, p.clamp_lo, p.clamp_hi);
+    } else if (ci.x == 1) {
+        if (p.need_clamp) epi_mid16<H, true>(v, pa, p.clamp_lo, p.clamp_hi, ci.y, ci.z);
+        else epi_mid16<H, false>(v, pa, p.clamp_lo, p.clamp_hi, ci.y, ci.z);
+    } else {
+        epi_general16<OUT, ZX, H>(p, v, pa, kc, zr0, zr1, zs0, zs1);
     }
 }
 
@@ -267,12 +293,14 @@ __device__ __forceinline__ void stage16(const ConvParams &p, const uint32_t (&v)
 
 template <int OUT, bool ZX, int H>
 __device__ __forceinline__ void epi_half(const ConvParams &p, uint32_t (&v)[32], uint32_t pa,
-                                         int mode, int32_t rmid, int kc, int64_t m, bool row_ok,
+                                         int4 cinfo, int kc, int64_t m, bool row_ok,
                                          int zr0, int zr1, int zs0, int zs1) {
-    if (mode == 0) epi_fast16<H>(v, pa, p.clamp_lo, p.clamp_hi);
-    else if (mode == 1) epi_mid16<H>(v, pa, p.clamp_lo, p.clamp_hi, rmid);
-    else epi_general16<OUT, ZX, H>(p, v, pa, kc - H, zr0, zr1, zs0, zs1);
+    epi_requant16<OUT, ZX, H>(p, v, pa, cinfo, kc - H, zr0, zr1, zs0, zs1);
     if (row_ok) store16<OUT, H>(p, v, kc, m);
+}
+
+__device__ __forceinline__ void trace_ev(const ConvParams &p, int ev, int seq) {
+    if (p.trace != nullptr && blockIdx.x == 0 && seq < 1024) p.trace[ev * 1024 + seq] = globaltimer_ns();
 }
 
 // ------------------------------------------------------------------ the kernel
@@ -295,7 +323,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
     uint64_t *tempty = bars + 3 * NS + 2;   // [2]  epilogue -> MMA
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 4);
     EpiCol *par = reinterpret_cast<EpiCol *>(smem + p.off_par);
-    uint8_t *chunk_fast = smem + p.off_par + 16 * kMaxBN;   // [8] per 32-column chunk
+    int4 *chunk_info = reinterpret_cast<int4 *>(smem + p.off_par + 16 * kMaxBN);  // [8] {mode, rhiT, shT, 0}
 
     if (warp == kWarpTMA && lane == 0) {
         tma_prefetch_desc(&xmap);
@@ -319,12 +347,15 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
     const uint32_t tmem_base = *tmem_slot;
     const int taps_per_r = p.S * p.chunks;
 
-    if (warp == kWarpTMA) {
-        // ===================== TMA producer (one thread) =====================
+    if (warp == kWarpTMA || warp == 2 || warp == 3) {
+        // ===================== TMA producers (lane 0 of warps 0, 2, 3) =====================
+        // Each TMA issue costs the issuing thread a few hundred cycles (measured on B200:
+        // ~300-420 cycles per wait+expect_tx+load sequence, independent of box size up to
+        // 16 KB), so K-stages are dealt round-robin to kNumProducers threads.
         if (lane == 0) {
-            int stage = 0;
-            uint32_t phase = 0;
+            const int pi = warp == kWarpTMA ? 0 : warp - 1;       // 0, 1, 2
             const uint32_t tx = static_cast<uint32_t>(kBM * (p.pair ? 32 : p.bkp) + p.BN * p.BK);
+            int g = 0;                                              // CTA-local K-stage counter
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
                 const int m0 = (tile / p.n_tiles_n) * kBM;
                 const int n0 = (tile % p.n_tiles_n) * p.BN;
@@ -334,15 +365,22 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 const int q0 = rem - p0 * p.Q;
                 const int wb = q0 * p.stride_w - p.pad_w;
                 const int hb = p0 * p.stride_h - p.pad_h;
-                if (p.pair) {
-                    const int RS = p.R * p.S;
-                    for (int kb = 0; kb < p.num_kb; ++kb) {
+                for (int kb = 0; kb < p.num_kb; ++kb, ++g) {
+                    if (g % kNumProducers != pi) continue;
+                    const int stage = g % NS;
+                    const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
+                    mbar_wait(&empty[stage], phase ^ 1u);
+                    trace_ev(p, 0, g);
+                    const bool skip_b = (p.exp_flags & 1) && tile != static_cast<int>(blockIdx.x) && g >= NS;
+                    const bool skip_a = (p.exp_flags & 2) && tile != static_cast<int>(blockIdx.x) && g >= NS;
+                    mbar_arrive_expect_tx(&full[stage], (skip_b ? tx - static_cast<uint32_t>(p.BN * p.BK) : tx) -
+                                                            (skip_a ? static_cast<uint32_t>(kBM * p.bkp) : 0u));
+                    if (p.pair) {
+                        const int RS = p.R * p.S;
                         const int t0 = 2 * kb, t1 = t0 + 1;
                         const int r0 = t0 / p.S, s0 = t0 - r0 * p.S;
                         int r1 = r0, s1 = s0, kg1 = RS * 16;        // odd tail: B slot OOB -> 0
                         if (t1 < RS) { r1 = t1 / p.S; s1 = t1 - r1 * p.S; kg1 = t1 * 16; }
-                        mbar_wait(&empty[stage], phase ^ 1u);
-                        mbar_arrive_expect_tx(&full[stage], tx);
                         uint8_t *adst = smem + p.off_a + stage * p.a_stage_bytes;
                         uint8_t *bdst = smem + p.off_b + stage * p.b_stage_bytes;
                         tma_load_im2col_4d(adst, &xmap, &full[stage], 0, wb, hb, img,
@@ -351,25 +389,21 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                                            static_cast<uint16_t>(s1 * p.dil_w), static_cast<uint16_t>(r1 * p.dil_h));
                         tma_load_2d(bdst, &wmap, &full[stage], t0 * 16, n0);
                         tma_load_2d(bdst + p.BN * 16, &wmap, &full[stage], kg1, n0);
-                        if (++stage == NS) { stage = 0; phase ^= 1u; }
+                    } else {
+                        const int r = kb / taps_per_r;
+                        const int rem2 = kb - r * taps_per_r;
+                        const int s = rem2 / p.chunks;
+                        const int ch = rem2 - s * p.chunks;
+                        uint8_t *adst = IS4 ? smem + p.off_stg + stage * p.stg_stage_bytes
+                                            : smem + p.off_a + stage * p.a_stage_bytes;
+                        if (!skip_a)
+                            tma_load_im2col_4d(adst, &xmap, &full[stage], ch * p.bkp, wb, hb, img,
+                                               static_cast<uint16_t>(s * p.dil_w),
+                                               static_cast<uint16_t>(r * p.dil_h));
+                        if (!skip_b)
+                            tma_load_2d(smem + p.off_b + stage * p.b_stage_bytes, &wmap, &full[stage],
+                                        (r * p.S + s) * p.C8 + ch * p.BK, n0);
                     }
-                    continue;
-                }
-                for (int kb = 0; kb < p.num_kb; ++kb) {
-                    const int r = kb / taps_per_r;
-                    const int rem2 = kb - r * taps_per_r;
-                    const int s = rem2 / p.chunks;
-                    const int ch = rem2 - s * p.chunks;
-                    mbar_wait(&empty[stage], phase ^ 1u);
-                    mbar_arrive_expect_tx(&full[stage], tx);
-                    uint8_t *adst = IS4 ? smem + p.off_stg + stage * p.stg_stage_bytes
-                                        : smem + p.off_a + stage * p.a_stage_bytes;
-                    tma_load_im2col_4d(adst, &xmap, &full[stage], ch * p.bkp, wb, hb, img,
-                                       static_cast<uint16_t>(s * p.dil_w),
-                                       static_cast<uint16_t>(r * p.dil_h));
-                    tma_load_2d(smem + p.off_b + stage * p.b_stage_bytes, &wmap, &full[stage],
-                                (r * p.S + s) * p.C8 + ch * p.BK, n0);
-                    if (++stage == NS) { stage = 0; phase ^= 1u; }
                 }
             }
         }
@@ -379,16 +413,19 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
             int stage = 0;
             uint32_t phase = 0;
             int it = 0;
+            int gstage = 0;
             const uint32_t sbo = 8u * static_cast<uint32_t>(p.BK);
             const int ksteps = p.BK / 32;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
                 const int buf = it & 1;
                 const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
                 mbar_wait(&tempty[buf], acc_phase ^ 1u);
+                trace_ev(p, 2, it);
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
                 for (int kb = 0; kb < p.num_kb; ++kb) {
                     mbar_wait(IS4 ? &aready[stage] : &full[stage], phase);
+                    trace_ev(p, 3, gstage++);
                     tc_fence_after();
                     const uint32_t a_addr = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
                     const uint32_t b_addr = smem_u32(smem + p.off_b + stage * p.b_stage_bytes);
@@ -402,13 +439,15 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                         for (int k = 0; k < ksteps; ++k) {
                             const uint64_t ad = make_smem_desc(a_addr + 32u * k, 16u, sbo, p.sw_layout);
                             const uint64_t bd = make_smem_desc(b_addr + 32u * k, 16u, sbo, p.sw_layout);
-                            mma_i8(d_tmem, ad, bd, p.idesc, (kb | k) != 0 ? 1u : 0u);
+                            if (!(p.exp_flags & 4) || (kb | k) == 0)
+                                mma_i8(d_tmem, ad, bd, p.idesc, (kb | k) != 0 ? 1u : 0u);
                         }
                     }
                     mma_commit(&empty[stage]);
                     if (++stage == NS) { stage = 0; phase ^= 1u; }
                 }
                 mma_commit(&tfull[buf]);
+                trace_ev(p, 4, it);
             }
         }
     } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kNumEpiWarps) {
@@ -420,7 +459,6 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
         const uint32_t par_base = smem_u32(par);
         const int nchunks = (p.BN + 31) / 32;
         const bool force_general = (OUT == OUT_S32) || ZX;
-        const int32_t rmid = 1 + 2 * p.y_zero;
         int cached_n0 = -1;
         int it = 0;
         const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
@@ -443,22 +481,24 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                     nn = __ldg(p.shift + k);
                 }
                 const bool all_fast = __ballot_sync(0xffffffffu, nn >= 33 && nn <= 52) == 0xffffffffu;
-                const bool all_mid =
-                    __ballot_sync(0xffffffffu, (nn >= 14 && nn <= 33) || k >= p.K) == 0xffffffffu;
+                const bool all_mid = __ballot_sync(0xffffffffu, nn >= 20 && nn <= 50) == 0xffffffffu;
                 const int mode = force_general ? 2 : (all_fast ? 0 : (all_mid ? 1 : 2));
+                const int T = max(33, __reduce_max_sync(0xffffffffu, nn));
                 if (OUT != OUT_S32 && k < p.K) {
                     if (mode == 0) {
                         e.c2 = (1 << (nn - 33)) + p.y_zero * (1 << (nn - 32));
                         e.c3 = nn - 32;
                     } else if (mode == 1) {
-                        e.c2 = 33 - nn;
-                        e.c3 = 1 << (nn - 20 > 0 ? nn - 20 : 0);
+                        e.c2 = T - nn;
+                        e.c3 = 1 << (nn - 20);
                     } else {
                         e.c2 = nn;
                     }
                 }
                 if (c < p.BN) *reinterpret_cast<EpiCol *>(reinterpret_cast<uint8_t *>(par) + 16 * c) = e;
-                if (lane == 0) chunk_fast[ew] = static_cast<uint8_t>(mode);
+                if (lane == 0)
+                    chunk_info[ew] = make_int4(mode, mode == 1 ? (1 << (T - 33)) + p.y_zero * (1 << (T - 32)) : 0,
+                                               T - 32, 0);
                 named_bar_sync(1, kNumEpiWarps * 32);
                 cached_n0 = n0;
             }
@@ -474,6 +514,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 valid_tap_range(qq, p.stride_w, p.pad_w, p.dil_w, p.W, p.S, zs0, zs1);
             }
             mbar_wait(&tfull[buf], acc_phase);
+            if (ew == 0 && lane == 0) trace_ev(p, 5, it);
             tc_fence_after();
             const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
                                    static_cast<uint32_t>(buf * p.BN);
@@ -486,27 +527,22 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 named_bar_sync(1, kNumEpiWarps * 32);
                 for (int ci = half; ci < nchunks; ci += 2) {
                     const int col0 = ci * 32;
+                    if (p.exp_flags & 16) continue;
                     __syncwarp();
                     tmem_ld_32x32b_x32(taddr + col0, v);
                     tmem_wait_ld();
+                    if (p.exp_flags & 8) { if (v[0] == 0x12345) asm volatile("trap;"); continue; }
                     const uint32_t pa = par_base + 16u * col0;
-                    const int mode = chunk_fast[ci];
-                    if (mode == 0) {
-                        epi_fast16<0>(v, pa, p.clamp_lo, p.clamp_hi);
-                        epi_fast16<16>(v, pa, p.clamp_lo, p.clamp_hi);
-                    } else if (mode == 1) {
-                        epi_mid16<0>(v, pa, p.clamp_lo, p.clamp_hi, rmid);
-                        epi_mid16<16>(v, pa, p.clamp_lo, p.clamp_hi, rmid);
-                    } else {
-                        epi_general16<OUT, ZX, 0>(p, v, pa, n0 + col0, zr0, zr1, zs0, zs1);
-                        epi_general16<OUT, ZX, 16>(p, v, pa, n0 + col0, zr0, zr1, zs0, zs1);
-                    }
+                    const int4 cinfo = chunk_info[ci];
+                    epi_requant16<OUT, ZX, 0>(p, v, pa, cinfo, n0 + col0, zr0, zr1, zs0, zs1);
+                    epi_requant16<OUT, ZX, 16>(p, v, pa, cinfo, n0 + col0, zr0, zr1, zs0, zs1);
                     stage16<OUT, 0>(p, v, ystg_base, row, col0);
                     stage16<OUT, 16>(p, v, ystg_base, row, col0 + 16);
                 }
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&tempty[buf]);    // accumulator drained: MMA may reuse it
+                if (ew == 0 && lane == 0) trace_ev(p, 6, it);
                 fence_proxy_async_smem();
                 named_bar_sync(1, kNumEpiWarps * 32);
                 if (storer) {
@@ -515,6 +551,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                         tma_store_2d(&ymap, smem + p.off_ystg + g * 128 * p.y_gw,
                                      n0 * kBits / 8 + g * p.y_gw, m0);
                     bulk_commit();
+                    trace_ev(p, 7, it);
                 }
                 continue;
             } else {
@@ -526,10 +563,10 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                     else tmem_ld_32x32b_x16(taddr + col0, v);
                     tmem_wait_ld();
                     const uint32_t pa = par_base + 16u * col0;
-                    const int mode = chunk_fast[ci];
-                    epi_half<OUT, ZX, 0>(p, v, pa, mode, rmid, n0 + col0, m, row_ok, zr0, zr1, zs0, zs1);
+                    const int4 cinfo = chunk_info[ci];
+                    epi_half<OUT, ZX, 0>(p, v, pa, cinfo, n0 + col0, m, row_ok, zr0, zr1, zs0, zs1);
                     if (nc == 32)
-                        epi_half<OUT, ZX, 16>(p, v, pa, mode, rmid, n0 + col0 + 16, m, row_ok, zr0, zr1, zs0, zs1);
+                        epi_half<OUT, ZX, 16>(p, v, pa, cinfo, n0 + col0 + 16, m, row_ok, zr0, zr1, zs0, zs1);
                 }
             }
             tc_fence_before();
@@ -540,6 +577,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
     } else if (IS4 && warp >= kWarpCvt0 && warp < kWarpCvt0 + kNumCvtWarps) {
         // ===================== int4 -> int8 widening (4 warps) =====================
         const int ct = (warp - kWarpCvt0) * 32 + lane;      // 0..127
+        int cstage = 0;
         const int cshift = p.cvt_shift;                      // log2(16-byte packed chunks/pixel)
         const int nchunks = kBM << cshift;
         const bool sgn = ((p.idesc >> 7) & 1u) != 0;
@@ -550,6 +588,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
             for (int kb = 0; kb < p.num_kb; ++kb) {
                 mbar_wait(&full[stage], phase);
+                if (ct == 0) trace_ev(p, 8, cstage++);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
                 for (int g = ct; g < nchunks; g += kNumCvtWarps * 32) {
@@ -578,6 +617,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 fence_proxy_async_smem();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&aready[stage]);
+                if (ct == 0) trace_ev(p, 9, cstage - 1);
                 if (++stage == NS) { stage = 0; phase ^= 1u; }
             }
         }

@@ -69,12 +69,15 @@ __device__ __forceinline__ bool mbar_try_wait_sleep(uint32_t addr, uint32_t pari
 // suspended (1 ms hint) until the phase completes, so idle roles do not steal
 // issue slots from working warps.  A wait longer than ~4 s traps (a protocol
 // bug becomes a launch error instead of a hang).
+#ifndef QC_WAIT_SLEEP
+#define QC_WAIT_SLEEP 0
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     const uint32_t a = smem_u32(bar);
     if (mbar_try_wait(a, parity)) return;
     uint64_t t0 = 0;
     uint32_t it = 0;
-    while (!mbar_try_wait_sleep(a, parity)) {
+    while (!(QC_WAIT_SLEEP ? mbar_try_wait_sleep(a, parity) : mbar_try_wait(a, parity))) {
         if ((++it & 63u) == 0) {
             const uint64_t t = globaltimer_ns();
             if (t0 == 0) t0 = t;

@@ -12,6 +12,9 @@
 #include <cstdint>
 #include <cstring>
 #include <mutex>
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
 
 #include "qconv.h"
 #include "conv_fwd.cuh"
@@ -226,10 +229,10 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
                        (static_cast<int64_t>(d->k) * ybits / 8) % 16 == 0 &&
                        (y_gw == 32 || y_gw == 64 || (y_gw == 128 && tile_row_bytes % 128 == 0));
     const uint32_t ystg_bytes = y_tma ? 128u * static_cast<uint32_t>(tile_row_bytes) : 0u;
-    const uint32_t fixed = static_cast<uint32_t>(qc::kMaxBN) * 16u + 64u + 1024u + ystg_bytes;
+    const uint32_t fixed = static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 1024u + ystg_bytes;
     const uint32_t budget = 227u * 1024u - 1024u - fixed;
     int stages = static_cast<int>(budget / per_stage);
-    stages = std::min(stages, 8);
+    stages = std::min(stages, 32);     // deep rings: TMA latency is ~1-3 us under load
     if (stages < 2) return QC_ERR_UNSUPPORTED;
     pl->stages = stages;
     qc::ConvParams &p = pl->cp;
@@ -243,7 +246,7 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.y_gmask = y_gw == 128 ? 7 : (y_gw == 64 ? 3 : 1);
     p.n_ygroups = y_tma ? tile_row_bytes / y_gw : 0;
     p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + ystg_bytes, 16));
-    p.off_bar = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 64u, 8));
+    p.off_bar = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u, 8));
     const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 4) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;       // + alignment slack for the 1024-B base
     pl->grid = std::min(pl->num_tiles, sms);
@@ -278,6 +281,7 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.sw_layout = pl->BK == 128 ? 2 : (pl->BK == 64 ? 4 : 6);
     p.pair = pair ? 1 : 0;
     p.cvt_shift = pl->bkp >= 64 ? 2 : (pl->bkp >= 32 ? 1 : 0);
+    p.need_clamp = (d->y_t != QC_S32 && (d->clamp_lo > dtype_min(d->y_t) || d->clamp_hi < dtype_max(d->y_t))) ? 1 : 0;
     p.sw_mask = pl->BK == 128 ? 7 : (pl->BK == 64 ? 3 : 1);
     p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), dtype_signed(d->x_t), dtype_signed(d->w_t));
     p.tmem_cols = pl->tmem_cols;
@@ -367,8 +371,29 @@ qc_status launch_conv_t(const Plan &pl, const CUtensorMap &xm, const CUtensorMap
     cfg.stream = stream;
     cfg.attrs = nullptr;
     cfg.numAttrs = 0;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, pl.cp);
+    // debug tracing (QC_TRACE=<file>): timestamps of CTA 0's pipeline events, dumped after a sync
+    static const char *trace_file = std::getenv("QC_TRACE");
+    static const char *exp_env = std::getenv("QC_EXPERIMENT");
+    qc::ConvParams cp = pl.cp;
+    cp.exp_flags = exp_env ? std::atoi(exp_env) : 0;
+    unsigned long long *tbuf = nullptr;
+    if (trace_file) {
+        cudaMalloc(&tbuf, 16 * 1024 * sizeof(unsigned long long));
+        cudaMemsetAsync(tbuf, 0, 16 * 1024 * sizeof(unsigned long long), stream);
+        cp.trace = tbuf;
+    }
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
     if (e != cudaSuccess) return cuda_fail(e);
+    if (tbuf) {
+        std::vector<unsigned long long> h(16 * 1024);
+        cudaMemcpyAsync(h.data(), tbuf, h.size() * 8, cudaMemcpyDeviceToHost, stream);
+        cudaStreamSynchronize(stream);
+        cudaFree(tbuf);
+        if (FILE *f = std::fopen(trace_file, "ab")) {
+            std::fwrite(h.data(), 8, h.size(), f);
+            std::fclose(f);
+        }
+    }
     return QC_OK;
 }
 
