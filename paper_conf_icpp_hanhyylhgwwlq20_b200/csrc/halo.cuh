@@ -1,0 +1,272 @@
+// halo.cuh -- "halo" variant of the implicit-GEMM conv for stride-1 convolutions.
+//
+// Same method as conv_fwd.cuh (Alg.2 P:L216-223 with the fused epilogue of
+// P:L223/P:L253/P:L265), different data movement, chosen for B200's TMA:
+//  * A tile = Rt whole output rows, each padded to Wh = W + 2*pad_w columns
+//    (columns >= Q are computed and discarded).  Instead of one im2col TMA per
+//    filter tap (R*S loads of 128 pixels, every input pixel fetched R*S times),
+//    ONE tiled TMA brings the (Rt+R-1) x Wh input halo of the tile, all channels,
+//    as 16-byte channel planes [plane][row][col][16 B] (zero-filled outside the
+//    image = the padding).  Every tap (r, s) is then the same buffer read at a
+//    pixel offset r*Wh + s: the UMMA no-swizzle K-major descriptor takes
+//    start = plane + (r*Wh+s)*16, SBO = 128 (8 pixels), LBO = plane stride.
+//  * B (weights of the CTA's N tile) is resident in shared memory for the whole
+//    kernel, loaded by one TMA as [K-chunk plane][BN rows][16 B].
+//  * The C=16 space-to-depth stem pairs taps (r,s),(r,s+1) in one K=32 MMA
+//    (LBO = 16: the next tap is the next pixel).
+// The paper's precomputed-offset gather and register prefetch
+// have no counterpart: the hardware gathers, shared memory reuses.
+#pragma once
+#include "conv_fwd.cuh"
+
+namespace qc {
+
+template <bool IS4, int OUT>
+__global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
+qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap bmap,
+                  const __grid_constant__ CUtensorMap ymap, const __grid_constant__ ConvParams p) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                                ~uintptr_t(1023));
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    const int NS = p.stages;
+
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + p.off_bar);
+    uint64_t *hfull = bars;                 // [NS] halo TMA -> (converter | MMA)
+    uint64_t *hempty = bars + NS;           // [NS] MMA -> producer
+    uint64_t *hready = bars + 2 * NS;       // [NS] converter -> MMA (4-bit)
+    uint64_t *tfull = bars + 3 * NS;        // [2]
+    uint64_t *tempty = bars + 3 * NS + 2;   // [2]
+    uint64_t *bfull = bars + 3 * NS + 4;    // [1] resident weights landed
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 5);
+    EpiCol *par = reinterpret_cast<EpiCol *>(smem + p.off_par);
+    int4 *chunk_info = reinterpret_cast<int4 *>(smem + p.off_par + 16 * kMaxBN);
+
+    if (warp == kWarpTMA && lane == 0) {
+        tma_prefetch_desc(&hmap);
+        tma_prefetch_desc(&bmap);
+        tma_prefetch_desc(&ymap);
+        for (int i = 0; i < NS; ++i) {
+            mbar_init(&hfull[i], 1);
+            mbar_init(&hempty[i], 1);
+            mbar_init(&hready[i], kNumCvtWarps);
+        }
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(&tfull[i], 1);
+            mbar_init(&tempty[i], kNumEpiWarps);
+        }
+        mbar_init(bfull, 1);
+        fence_mbar_init();
+    }
+    if (warp == kWarpMMA) tmem_alloc(tmem_slot, p.tmem_cols);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    // all tiles of this CTA share one N tile (grid is a multiple of n_tiles_n)
+    const int n0 = (static_cast<int>(blockIdx.x) % p.n_tiles_n) * p.BN;
+
+    if (warp == kWarpTMA) {
+        // ===================== TMA producer =====================
+        if (lane == 0) {   // one thread issues (measured faster than an elected warp-wide loop)
+            constexpr bool leader = true;
+            if (leader) mbar_arrive_expect_tx(bfull, p.b_res_bytes);
+            if (leader) tma_load_3d(smem + p.off_bres, &bmap, bfull, 0, n0, 0);
+            int g = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
+                const int mt = tile / p.n_tiles_n;
+                const int img = mt / p.tiles_per_img;
+                const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
+                const int stage = g % NS;
+                const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
+                mbar_wait(&hempty[stage], phase ^ 1u);
+                if (leader) trace_ev(p, 0, g);
+                if (leader) mbar_arrive_expect_tx(&hfull[stage], p.halo_tx);
+                uint8_t *dst = IS4 ? smem + p.off_hp + stage * p.hp_stage_bytes
+                                   : smem + p.off_hx + stage * p.hx_stage_bytes;
+                if (leader) tma_load_5d(dst, &hmap, &hfull[stage], 0, -p.pad_w, p0 - p.pad_h, img, 0);
+            }
+        }
+    } else if (warp == kWarpMMA) {
+        // ===================== MMA issuer =====================
+        if (lane == 0) {   // one thread issues (measured faster than an elected warp-wide loop)
+            constexpr bool leader = true;
+            // per-MMA descriptor offsets (16-byte units), built once: K order = (r, s, plane pair)
+            uint2 *mtab = reinterpret_cast<uint2 *>(smem + p.off_mtab);
+            const uint32_t bplane = static_cast<uint32_t>(p.BN) * 16u;
+            {
+                int i = 0;
+                for (int r = 0; r < p.R; ++r)
+                    for (int s = 0; s < p.S; s += (p.tap_pair ? 2 : 1))
+                        for (int j = 0; j < (p.tap_pair ? 1 : p.nplanes); j += 2, ++i) {
+                            const uint32_t aoff = static_cast<uint32_t>(r * p.Wh + s) * 16u +
+                                                  static_cast<uint32_t>(j) * p.h_plane_bytes;
+                            const uint32_t boff = static_cast<uint32_t>(
+                                (p.tap_pair ? (r * p.S + s) : ((r * p.S + s) * p.nplanes + j))) * bplane;
+                            mtab[i] = make_uint2(aoff >> 4, boff >> 4);
+                        }
+            }
+            const int nmma = p.n_mma;
+            const uint64_t bdesc0 = make_smem_desc(smem_u32(smem + p.off_bres), bplane, 128u, 0u);
+            const uint32_t a_lbo = p.tap_pair ? 16u : p.h_plane_bytes;
+            mbar_wait(bfull, 0);
+            tc_fence_after();
+            int it = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+                const int buf = it & 1;
+                const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
+                const int stage = it % NS;
+                const uint32_t phase = static_cast<uint32_t>(it / NS) & 1u;
+                mbar_wait(&tempty[buf], acc_phase ^ 1u);
+                if (leader) trace_ev(p, 2, it);
+                tc_fence_after();
+                mbar_wait(IS4 ? &hready[stage] : &hfull[stage], phase);
+                if (leader) trace_ev(p, 3, it);
+                tc_fence_after();
+                const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
+                const uint64_t adesc0 = make_smem_desc(smem_u32(smem + p.off_hx + stage * p.hx_stage_bytes),
+                                                       a_lbo, 128u, 0u);
+                for (int i = 0; i < nmma; ++i) {
+                    const uint2 o = mtab[i];
+                    mma_i8(d_tmem, adesc0 + o.x, bdesc0 + o.y, p.idesc, i > 0 ? 1u : 0u);
+                }
+                if (leader) mma_commit(&hempty[stage]);
+                if (leader) mma_commit(&tfull[buf]);
+                if (leader) trace_ev(p, 4, it);
+            }
+        }
+    } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kNumEpiWarps) {
+        // ===================== epilogue =====================
+        const int ew = warp - kWarpEpi0;
+        const int quarter = warp & 3;
+        const int half = ew >> 2;
+        const int row = quarter * 32 + lane;           // accumulator row = padded output index
+        const int rr = row / p.Wh;
+        const int qq = row - rr * p.Wh;
+        const bool row_ok = rr < p.Rt && qq < p.Q;      // rows beyond P are clipped by the Y map
+        const int srow = rr * p.Q + qq;                 // row inside the [Rt][Q] staging box
+        const uint32_t par_base = smem_u32(par);
+        const int nchunks = p.BN / 32;
+        const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
+        fill_epilogue_params<OUT>(p, par, chunk_info, n0, ew, lane, false);
+        int it = 0;
+        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+            const int buf = it & 1;
+            const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
+            const int mt = tile / p.n_tiles_n;
+            const int img = mt / p.tiles_per_img;
+            const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
+            mbar_wait(&tfull[buf], acc_phase);
+            if (ew == 0 && lane == 0) trace_ev(p, 5, it);
+            tc_fence_after();
+            const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
+                                   static_cast<uint32_t>(buf * p.BN);
+            const bool storer = ew == 0 && lane == 0;
+            if (storer) bulk_wait_read<1>();
+            named_bar_sync(1, kNumEpiWarps * 32);
+            const uint32_t ystg_it = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes;
+            // TMEM loads double-buffered: chunk ci+2 is in flight while chunk ci is requantized
+            uint32_t va[32], vb[32];
+            auto process = [&](uint32_t (&v)[32], int ci) {
+                const int col0 = ci * 32;
+                const uint32_t pa = par_base + 16u * col0;
+                const int4 cinfo = chunk_info[ci];
+                epi_requant16<OUT, false, 0>(p, v, pa, cinfo, n0 + col0, 0, 0, 0, 0);
+                epi_requant16<OUT, false, 16>(p, v, pa, cinfo, n0 + col0, 0, 0, 0, 0);
+                if (row_ok) {
+                    stage16<OUT, 0>(p, v, ystg_it, srow, col0);
+                    stage16<OUT, 16>(p, v, ystg_it, srow, col0 + 16);
+                }
+            };
+            if (!IS4) {   // 8-bit kernels (384 threads) have the registers to double-buffer
+                __syncwarp();
+                if (half < nchunks) tmem_ld_32x32b_x32(taddr + half * 32, va);
+                for (int ci = half; ci < nchunks; ci += 4) {
+                    tmem_wait_ld();
+                    __syncwarp();
+                    if (ci + 2 < nchunks) tmem_ld_32x32b_x32(taddr + (ci + 2) * 32, vb);
+                    process(va, ci);
+                    if (ci + 2 >= nchunks) break;
+                    tmem_wait_ld();
+                    __syncwarp();
+                    if (ci + 4 < nchunks) tmem_ld_32x32b_x32(taddr + (ci + 4) * 32, va);
+                    process(vb, ci + 2);
+                }
+            } else {
+                for (int ci = half; ci < nchunks; ci += 2) {
+                    __syncwarp();
+                    tmem_ld_32x32b_x32(taddr + ci * 32, va);
+                    tmem_wait_ld();
+                    process(va, ci);
+                }
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&tempty[buf]);
+            if (ew == 0 && lane == 0) trace_ev(p, 6, it);
+            fence_proxy_async_smem();
+            named_bar_sync(1, kNumEpiWarps * 32);
+            if (storer) {
+                constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
+                for (int gi = 0; gi < p.n_ygroups; ++gi)
+                    tma_store_4d(&ymap, smem + p.off_ystg + (it & 1) * p.ystg_bytes + gi * 128 * p.y_gw,
+                                 n0 * kBits / 8 + gi * p.y_gw, 0, p0, img);
+                bulk_commit();
+            }
+        }
+        if (ew == 0 && lane == 0) bulk_wait<0>();
+    } else if (IS4 && warp >= kWarpCvt0 && warp < kWarpCvt0 + kNumCvtWarps) {
+        // ===================== int4 -> int8 plane widening =====================
+        // packed plane j (16 B = 32 channels per pixel) -> int8 planes 2j (channels 0..15)
+        // and 2j+1 (16..31) at the same pixel offset
+        const int ct = (warp - kWarpCvt0) * 32 + lane;
+        const bool sgn = ((p.idesc >> 7) & 1u) != 0;
+        const int npix = p.HR * p.Wh;
+        const int nchunks = npix * (p.nplanes / 2);
+        int g = 0;
+        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
+            const int stage = g % NS;
+            const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
+            mbar_wait(&hfull[stage], phase);
+            if (ct == 0) trace_ev(p, 8, g);
+            const uint32_t src = smem_u32(smem + p.off_hp + stage * p.hp_stage_bytes);
+            const uint32_t dst = smem_u32(smem + p.off_hx + stage * p.hx_stage_bytes);
+            for (int c = ct; c < nchunks; c += kNumCvtWarps * 32) {
+                const int j = c / npix;
+                const int px = c - j * npix;
+                const uint4 pk = lds128u(src + static_cast<uint32_t>(c) * 16u);
+                const uint32_t s4[4] = {pk.x, pk.y, pk.z, pk.w};
+                uint32_t o[8];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    uint32_t lo = s4[i] & 0x0F0F0F0Fu;
+                    uint32_t hi = (s4[i] >> 4) & 0x0F0F0F0Fu;
+                    if (sgn) {
+                        lo = ((lo ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
+                        hi = ((hi ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
+                    }
+                    o[2 * i] = __byte_perm(lo, hi, 0x5140);
+                    o[2 * i + 1] = __byte_perm(lo, hi, 0x7362);
+                }
+                const uint32_t d0 = dst + static_cast<uint32_t>(2 * j) * p.h_plane_bytes + static_cast<uint32_t>(px) * 16u;
+                sts128(d0, o[0], o[1], o[2], o[3]);
+                sts128(d0 + p.h_plane_bytes, o[4], o[5], o[6], o[7]);
+            }
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&hready[stage]);
+            if (ct == 0) trace_ev(p, 9, g);
+        }
+    }
+
+    tc_fence_before();
+    __syncthreads();
+    if (warp == kWarpMMA) {
+        __syncwarp();
+        tc_fence_after();
+        tmem_dealloc(tmem_base, p.tmem_cols);
+    }
+}
+
+}  // namespace qc

@@ -174,12 +174,14 @@ struct QuantS2DParams {
     int32_t z, qmin, qmax, bf16;
 };
 
+template <int C>   // C > 0: compile-time channel count (stem: 3); C == 0: runtime p.c
 __global__ void __launch_bounds__(256) quantize_s2d_kernel(const __grid_constant__ QuantS2DParams p) {
     QuantParams qp;
     qp.x = p.x; qp.inv_s = p.inv_s; qp.flo = p.flo; qp.fhi = p.fhi;
     qp.z = p.z; qp.qmin = p.qmin; qp.qmax = p.qmax; qp.bf16 = p.bf16;
+    const int32_t c = C > 0 ? C : p.c;
     const int64_t total = static_cast<int64_t>(p.n) * p.hs * p.ws;
-    const int32_t c4 = 4 * p.c;
+    const int32_t c4 = 4 * c;
     for (int64_t t = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; t < total;
          t += static_cast<int64_t>(gridDim.x) * blockDim.x) {
         const int64_t img = t / (static_cast<int64_t>(p.hs) * p.ws);
@@ -193,15 +195,61 @@ __global__ void __launch_bounds__(256) quantize_s2d_kernel(const __grid_constant
                 const int32_t ch = ch0 + jj;
                 int32_t code = p.z;
                 if (ch < c4) {
-                    const int32_t blk = ch / p.c, cc = ch - blk * p.c;
+                    const int32_t blk = ch / c, cc = ch - blk * c;
                     const int32_t hh = 2 * i + (blk >> 1) - p.pad_h;
                     const int32_t ww = 2 * j + (blk & 1) - p.pad_w;
                     if (hh >= 0 && hh < p.h && ww >= 0 && ww < p.w)
-                        code = quantize_one(load_x(qp, ((img * p.h + hh) * p.w + ww) * p.c + cc), qp);
+                        code = quantize_one(load_x(qp, ((img * p.h + hh) * p.w + ww) * c + cc), qp);
                 }
                 w[jj >> 2] |= static_cast<uint32_t>(code & 0xFF) << (8 * (jj & 3));
             }
             *reinterpret_cast<uint4 *>(dst + ch0) = make_uint4(w[0], w[1], w[2], w[3]);
+        }
+    }
+}
+
+// Row-blocked variant for 4c <= 16 and w*c <= 4096: one CTA per (image, output row i)
+// stages the two input rows 2i-pad_h, 2i+1-pad_h in shared memory with coalesced 16-byte
+// loads, then thread j emits the 16 codes of X2[n, i, j, :] as one 16-byte store.
+__global__ void __launch_bounds__(128) quantize_s2d_rows_kernel(const __grid_constant__ QuantS2DParams p) {
+    __shared__ __align__(16) float rows[2][4096];
+    QuantParams qp;
+    qp.x = p.x; qp.inv_s = p.inv_s; qp.flo = p.flo; qp.fhi = p.fhi;
+    qp.z = p.z; qp.qmin = p.qmin; qp.qmax = p.qmax; qp.bf16 = p.bf16;
+    const int32_t rowlen = p.w * p.c;
+    for (int64_t blk = blockIdx.x; blk < static_cast<int64_t>(p.n) * p.hs; blk += gridDim.x) {
+        const int64_t img = blk / p.hs;
+        const int32_t i = static_cast<int32_t>(blk - img * p.hs);
+        __syncthreads();
+        for (int b = 0; b < 2; ++b) {
+            const int32_t hh = 2 * i + b - p.pad_h;
+            if (hh < 0 || hh >= p.h) continue;
+            const int64_t base = (img * p.h + hh) * rowlen;
+            if (!p.bf16 && (rowlen % 4) == 0) {
+                const float4 *src = reinterpret_cast<const float4 *>(static_cast<const float *>(p.x) + base);
+                for (int t = threadIdx.x; t < rowlen / 4; t += blockDim.x)
+                    reinterpret_cast<float4 *>(rows[b])[t] = __ldg(src + t);
+            } else {
+                for (int t = threadIdx.x; t < rowlen; t += blockDim.x) rows[b][t] = load_x(qp, base + t);
+            }
+        }
+        __syncthreads();
+        for (int32_t j = threadIdx.x; j < p.ws; j += blockDim.x) {
+            uint32_t wv[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+            for (int jj = 0; jj < 16; ++jj) {
+                int32_t code = p.z;
+                if (jj < 4 * p.c) {
+                    const int32_t blkc = jj / p.c, cc = jj - blkc * p.c;
+                    const int32_t hh = 2 * i + (blkc >> 1) - p.pad_h;
+                    const int32_t ww = 2 * j + (blkc & 1) - p.pad_w;
+                    if (hh >= 0 && hh < p.h && ww >= 0 && ww < p.w)
+                        code = quantize_one(rows[blkc >> 1][ww * p.c + cc], qp);
+                }
+                wv[jj >> 2] |= static_cast<uint32_t>(code & 0xFF) << (8 * (jj & 3));
+            }
+            *reinterpret_cast<uint4 *>(p.y + ((img * p.hs + i) * p.ws + j) * 16) =
+                make_uint4(wv[0], wv[1], wv[2], wv[3]);
         }
     }
 }

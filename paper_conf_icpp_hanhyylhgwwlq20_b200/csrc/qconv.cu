@@ -19,6 +19,7 @@
 #include "qconv.h"
 #include "conv_fwd.cuh"
 #include "prep.cuh"
+#include "halo.cuh"
 
 namespace {
 
@@ -228,7 +229,8 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const bool y_tma = d->y_t != QC_S32 && BN % 32 == 0 &&
                        (static_cast<int64_t>(d->k) * ybits / 8) % 16 == 0 &&
                        (y_gw == 32 || y_gw == 64 || (y_gw == 128 && tile_row_bytes % 128 == 0));
-    const uint32_t ystg_bytes = y_tma ? 128u * static_cast<uint32_t>(tile_row_bytes) : 0u;
+    const uint32_t ystg_one = y_tma ? 128u * static_cast<uint32_t>(tile_row_bytes) : 0u;
+    const uint32_t ystg_bytes = 2u * ystg_one;   // double-buffered
     const uint32_t fixed = static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 1024u + ystg_bytes;
     const uint32_t budget = 227u * 1024u - 1024u - fixed;
     int stages = static_cast<int>(budget / per_stage);
@@ -241,6 +243,7 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.off_b = p.off_a + a_bytes * stages;
     p.off_stg = p.off_b + b_bytes * stages;
     p.off_ystg = static_cast<uint32_t>(align_up(p.off_stg + stg_bytes * stages, 1024));
+    p.ystg_bytes = ystg_one;
     p.y_tma = y_tma ? 1 : 0;
     p.y_gw = y_gw;
     p.y_gmask = y_gw == 128 ? 7 : (y_gw == 64 ? 3 : 1);
@@ -402,6 +405,200 @@ qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &
                       const CUtensorMap &ym, cudaStream_t stream) {
     return pl.cp.x_zero != 0 ? launch_conv_t<IS4, OUT, true>(pl, xm, wm, ym, stream)
                              : launch_conv_t<IS4, OUT, false>(pl, xm, wm, ym, stream);
+}
+
+// ------------------------------------------------------------------ halo mode (stride 1)
+bool halo_disabled() {
+    static const bool off = std::getenv("QC_NO_HALO") != nullptr;
+    return off;
+}
+
+// Decide whether the stride-1 halo kernel applies and fill its plan.
+bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
+    if (halo_disabled()) return false;
+    if (d->stride_h != 1 || d->stride_w != 1 || d->dil_h != 1 || d->dil_w != 1) return false;
+    if (d->x_zero != 0 || d->y_t == QC_S32) return false;
+    const bool is4 = g.bits == 4;
+    const int C8 = d->c;                                 // int8 bytes per pixel after widening
+    const bool tap_pair = !is4 && C8 == 16;
+    if (tap_pair) {
+        if (d->s % 2) return false;
+    } else if (C8 % 32) {
+        return false;
+    }
+    const int Wh = d->w + 2 * d->pad_w;
+    if (Wh > qc::kBM || Wh > 256) return false;
+    if (d->r * d->s == 1) return false;                 // no tap reuse: the im2col GEMM path is better
+    const int Rt = qc::kBM / Wh;
+    const int tpi = (g.P + Rt - 1) / Rt;
+    if (static_cast<double>(g.P) * g.Q / (static_cast<double>(tpi) * qc::kBM) < 0.7) return false;
+    const int HR = Rt + d->r - 1;
+    const int nplanes = C8 / 16;
+    const int nch = g.c_bytes / 16;                      // TMA channel chunks (packed for 4-bit)
+    if (nch < 1 || nch > 256 || HR > 256) return false;
+    const int KG8 = d->r * d->s * C8;
+    const int nK = KG8 / 16;
+    if (nK > 256) return false;
+    // N tile: largest of {round_up(K,32) <= 256, 128, 64, 32} whose weight slab fits in 100 KB
+    // the whole weight slab stays resident (one N tile): MMA issue costs ~75 cycles per
+    // instruction (measured), so narrower N tiles would be issue-bound
+    if (d->k > 256) return false;
+    const int BN = (d->k + 31) / 32 * 32;
+    if (static_cast<int64_t>(BN) * KG8 > 100 * 1024) return false;
+    const int ybits = dtype_bits(d->y_t);
+    const int tile_row_bytes = BN * ybits / 8;
+    const int y_gw = tile_row_bytes >= 128 ? 128 : tile_row_bytes;
+    if (!((static_cast<int64_t>(d->k) * ybits / 8) % 16 == 0 &&
+          (y_gw == 32 || y_gw == 64 || (y_gw == 128 && tile_row_bytes % 128 == 0))))
+        return false;
+    const int n_tiles_n = (d->k + BN - 1) / BN;
+    const int tiles_per_img = (g.P + Rt - 1) / Rt;
+    const int64_t num_tiles = static_cast<int64_t>(d->n) * tiles_per_img * n_tiles_n;
+    if (num_tiles > INT32_MAX) return false;
+    const uint32_t plane = static_cast<uint32_t>(HR * Wh * 16);
+    const uint32_t hx = static_cast<uint32_t>(align_up(static_cast<size_t>(nplanes) * plane, 1024));
+    const uint32_t hp = is4 ? static_cast<uint32_t>(align_up(static_cast<size_t>(nch) * plane, 1024)) : 0u;
+    const uint32_t bres = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * KG8, 1024));
+    const uint32_t ystg = 2u * 128u * static_cast<uint32_t>(tile_row_bytes);   // double-buffered
+    const uint32_t fixed = bres + ystg + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 2048u +
+                           8u * static_cast<uint32_t>(d->r * d->s * nplanes);
+    if (fixed + 2 * (hx + hp) > 227u * 1024u) return false;
+    int stages = static_cast<int>((227u * 1024u - fixed) / (hx + hp));
+    stages = std::min(stages, 6);
+    qc::ConvParams &p = pl->cp;
+    std::memset(&p, 0, sizeof(p));
+    p.M = static_cast<int32_t>(g.M);
+    p.P = g.P; p.Q = g.Q; p.PQ = g.P * g.Q; p.K = d->k;
+    p.BN = BN; p.n_tiles_n = n_tiles_n; p.num_tiles = static_cast<int32_t>(num_tiles);
+    p.S = d->s; p.R = d->r; p.H = d->h; p.W = d->w; p.C8 = C8;
+    p.stride_h = p.stride_w = 1; p.dil_h = p.dil_w = 1; p.pad_h = d->pad_h; p.pad_w = d->pad_w;
+    p.stages = stages;
+    p.Wh = Wh; p.Rt = Rt; p.HR = HR; p.tiles_per_img = tiles_per_img; p.nplanes = nplanes;
+    p.nk_planes = nK; p.tap_pair = tap_pair ? 1 : 0; p.h_plane_bytes = plane;
+    p.off_bres = 0;
+    p.b_res_bytes = static_cast<uint32_t>(BN) * static_cast<uint32_t>(KG8);
+    p.off_hx = bres;
+    p.hx_stage_bytes = hx;
+    p.off_hp = bres + hx * stages;
+    p.hp_stage_bytes = hp;
+    p.halo_tx = static_cast<uint32_t>(nch) * plane;
+    p.off_ystg = static_cast<uint32_t>(align_up(p.off_hp + hp * stages, 1024));
+    p.ystg_bytes = ystg / 2;
+    p.y_tma = 1;
+    p.y_gw = y_gw;
+    p.y_gmask = y_gw == 128 ? 7 : (y_gw == 64 ? 3 : 1);
+    p.n_ygroups = tile_row_bytes / y_gw;
+    p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + ystg, 16));
+    p.n_mma = tap_pair ? d->r * (d->s / 2) : d->r * d->s * (nplanes / 2);
+    p.off_mtab = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u, 16));
+    p.off_bar = static_cast<uint32_t>(align_up(p.off_mtab + 8u * static_cast<uint32_t>(p.n_mma), 8));
+    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 5) * 8 + 16);
+    pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
+    if (pl->smem_bytes > 227u * 1024u) return false;
+    p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), dtype_signed(d->x_t), dtype_signed(d->w_t));
+    pl->tmem_cols = pow2_cols(2 * BN);
+    p.tmem_cols = pl->tmem_cols;
+    p.y_zero = d->y_zero; p.clamp_lo = d->clamp_lo; p.clamp_hi = d->clamp_hi; p.x_zero = 0;
+    p.need_clamp = (d->clamp_lo > dtype_min(d->y_t) || d->clamp_hi < dtype_max(d->y_t)) ? 1 : 0;
+    p.y_row_bytes = static_cast<int64_t>(d->k) * ybits / 8;
+    const int sms = num_sms();
+    int grid = std::min<int64_t>(num_tiles, sms / n_tiles_n * n_tiles_n);
+    grid = std::max(grid / n_tiles_n * n_tiles_n, n_tiles_n);
+    pl->grid = grid;
+    pl->threads = is4 ? 512 : 384;
+    pl->BN = BN;
+    pl->n_tiles_n = n_tiles_n;
+    pl->num_tiles = static_cast<int>(num_tiles);
+    pl->stages = stages;
+    return true;
+}
+
+qc_status encode_halo_maps(const qconv_desc *d, const Geometry &g, const qc::ConvParams &p,
+                           const void *x, const void *w8, void *y, CUtensorMap *hm, CUtensorMap *bm,
+                           CUtensorMap *ym) {
+    const Driver &drv = driver();
+    if (!drv.tiled) return cuda_fail(drv.err);
+    const cuuint64_t cb = static_cast<cuuint64_t>(g.c_bytes);
+    {   // input halo: [chunk][n][h][w][16 B] view of NHWC
+        cuuint64_t dims[5] = {16, static_cast<cuuint64_t>(d->w), static_cast<cuuint64_t>(d->h),
+                              static_cast<cuuint64_t>(d->n), cb / 16};
+        cuuint64_t strides[4] = {cb, cb * d->w, cb * d->w * d->h, 16};
+        cuuint32_t box[5] = {16, static_cast<cuuint32_t>(p.Wh), static_cast<cuuint32_t>(p.HR), 1,
+                             static_cast<cuuint32_t>(cb / 16)};
+        cuuint32_t es[5] = {1, 1, 1, 1, 1};
+        CUresult r = drv.tiled(hm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 5, const_cast<void *>(x), dims, strides,
+                               box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+        small_tensor_fixup(hm, static_cast<uint64_t>(g.x_bytes));
+    }
+    {   // weights: [K-chunk][k][16 B] view of int8 KRSC
+        const cuuint64_t kg = static_cast<cuuint64_t>(d->r) * d->s * d->c;
+        cuuint64_t dims[3] = {16, static_cast<cuuint64_t>(d->k), kg / 16};
+        cuuint64_t strides[2] = {kg, 16};
+        cuuint32_t box[3] = {16, static_cast<cuuint32_t>(p.BN), static_cast<cuuint32_t>(kg / 16)};
+        cuuint32_t es[3] = {1, 1, 1};
+        CUresult r = drv.tiled(bm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, const_cast<void *>(w8), dims, strides,
+                               box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+        small_tensor_fixup(bm, static_cast<uint64_t>(g.w8_bytes));
+    }
+    {   // output: [n][p][q][k bytes], box [1][Rt][Q][y_gw]
+        const int yb = dtype_bits(d->y_t);
+        const cuuint64_t row = static_cast<cuuint64_t>(d->k) * yb / 8;
+        cuuint64_t dims[4] = {row, static_cast<cuuint64_t>(g.Q), static_cast<cuuint64_t>(g.P),
+                              static_cast<cuuint64_t>(d->n)};
+        cuuint64_t strides[3] = {row, row * g.Q, row * g.Q * g.P};
+        cuuint32_t box[4] = {static_cast<cuuint32_t>(p.y_gw), static_cast<cuuint32_t>(g.Q),
+                             static_cast<cuuint32_t>(p.Rt), 1};
+        cuuint32_t es[4] = {1, 1, 1, 1};
+        CUresult r = drv.tiled(ym, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, y, dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_for(p.y_gw),
+                               CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+        small_tensor_fixup(ym, static_cast<uint64_t>(g.y_bytes));
+    }
+    return QC_OK;
+}
+
+template <bool IS4, int OUT>
+qc_status launch_halo(const Plan &pl, const CUtensorMap &hm, const CUtensorMap &bm,
+                      const CUtensorMap &ym, cudaStream_t stream) {
+    auto kern = qc::qconv_halo_kernel<IS4, OUT>;
+    static int configured = 0;
+    if (!configured) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+        if (e != cudaSuccess) return cuda_fail(e);
+        configured = 1;
+    }
+    cudaLaunchConfig_t cfg;
+    std::memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
+    cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
+    cfg.dynamicSmemBytes = pl.smem_bytes;
+    cfg.stream = stream;
+    static const char *trace_file = std::getenv("QC_TRACE");
+    qc::ConvParams cp = pl.cp;
+    unsigned long long *tbuf = nullptr;
+    if (trace_file) {
+        cudaMalloc(&tbuf, 16 * 1024 * sizeof(unsigned long long));
+        cudaMemsetAsync(tbuf, 0, 16 * 1024 * sizeof(unsigned long long), stream);
+        cp.trace = tbuf;
+    }
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, hm, bm, ym, cp);
+    if (e != cudaSuccess) return cuda_fail(e);
+    if (tbuf) {
+        std::vector<unsigned long long> h(16 * 1024);
+        cudaMemcpyAsync(h.data(), tbuf, h.size() * 8, cudaMemcpyDeviceToHost, stream);
+        cudaStreamSynchronize(stream);
+        cudaFree(tbuf);
+        if (FILE *f = std::fopen(trace_file, "ab")) {
+            std::fwrite(h.data(), 8, h.size(), f);
+            std::fclose(f);
+        }
+    }
+    return QC_OK;
 }
 
 }  // namespace
@@ -568,6 +765,26 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
         if (s != QC_OK) return s;
         w8 = workspace;
     }
+    {   // stride-1 convolutions: halo kernel (one tiled TMA per tile, resident weights)
+        Plan hp;
+        if (need_z == 0 && make_halo_plan(d, g, &hp)) {
+            hp.cp.bias = bias;
+            hp.cp.mult = multiplier;
+            hp.cp.shift = shift;
+            hp.cp.y = y;
+            alignas(64) CUtensorMap hm, bm, ym;
+            s = encode_halo_maps(d, g, hp.cp, x, w8, y, &hm, &bm, &ym);
+            if (s != QC_OK) return s;
+            const bool is4 = g.bits == 4;
+            switch (d->y_t) {
+                case QC_U8: return is4 ? launch_halo<true, qc::OUT_U8>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_U8>(hp, hm, bm, ym, st);
+                case QC_S8: return is4 ? launch_halo<true, qc::OUT_S8>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_S8>(hp, hm, bm, ym, st);
+                case QC_U4: return is4 ? launch_halo<true, qc::OUT_U4>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_U4>(hp, hm, bm, ym, st);
+                case QC_S4: return is4 ? launch_halo<true, qc::OUT_S4>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_S4>(hp, hm, bm, ym, st);
+                default: break;
+            }
+        }
+    }
     qc::ConvParams &p = pl.cp;
     if (need_z) {
         int32_t *table = reinterpret_cast<int32_t *>(static_cast<uint8_t *>(workspace) + need_w);
@@ -668,9 +885,14 @@ qc_status qconv_quantize_pack_s2d(const qconv_desc *d, const void *x, qc_ftype x
     p.flo = static_cast<float>(p.qmin - p.z - 1);
     p.fhi = static_cast<float>(p.qmax - p.z + 1);
     p.bf16 = xt == QC_BF16;
-    const int64_t total = static_cast<int64_t>(p.n) * p.hs * p.ws;
-    const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, static_cast<int64_t>(num_sms()) * 16));
-    qc::quantize_s2d_kernel<<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(p);
+    {
+        const int64_t total = static_cast<int64_t>(p.n) * p.hs * p.ws;
+        const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, static_cast<int64_t>(num_sms()) * 32));
+        if (p.c == 3)
+            qc::quantize_s2d_kernel<3><<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(p);
+        else
+            qc::quantize_s2d_kernel<0><<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(p);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e);
     return QC_OK;

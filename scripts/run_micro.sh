@@ -1,3 +1,3 @@
 #!/bin/bash
 mkdir -p gpurun_out
-./scripts/micro/tma_bench > gpurun_out/tma_bench3.txt 2>&1
+./scripts/micro/mma_bench > gpurun_out/mma_bench.txt 2>&1
