@@ -353,6 +353,70 @@ __device__ __forceinline__ void trace_ev(const ConvParams &p, int ev, int seq) {
 }
 
 // ------------------------------------------------------------------ the kernel
+// Widen one 32-bit word of eight packed 4-bit codes (element 2i in the low nibble of byte i)
+// into two words of eight int8 values.  The nibble split uses the FMA pipe (IMAD) where it
+// can, since the integer ALU pipe is half rate and is what bounds the converter warps:
+// lo = w & 0x0F0F0F0F (LOP3), hi = (w - lo) >> 4 (IMAD + IMAD.HI), two byte permutes.
+__device__ __forceinline__ void widen_word(uint32_t w, bool sgn, uint32_t &o0, uint32_t &o1) {
+    uint32_t lo = w & 0x0F0F0F0Fu;
+    uint32_t hi = __umulhi(w - lo, 0x10000000u);
+    if (sgn) {          // sign-extend each nibble: ((v ^ 8) + 0x78) ^ 0x80 per byte
+        lo = ((lo ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
+        hi = ((hi ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
+    }
+    o0 = __byte_perm(lo, hi, 0x5140);
+    o1 = __byte_perm(lo, hi, 0x7362);
+}
+
+// int4 -> int8 widening of one staged operand tile (Sec.3.2 P:L231-235 bit unpacking,
+// done on chip): 16-byte packed chunk g of row g>>cshift becomes 32 widened bytes, written
+// with the 128B/64B/32B swizzle the MMA descriptor expects.  A thread's chunks are kStride
+// apart, i.e. (kStride >> cshift) >= 32 rows apart, so their swizzle phase is the same and
+// the destination offsets are computed once.  Four chunks are loaded before any is
+// converted so the shared-memory latency overlaps.
+__device__ __forceinline__ void widen_stage(uint32_t stg, uint32_t adst, int ct, int nchunks,
+                                            int cshift, uint32_t bkb, uint32_t sw, bool sgn) {
+    constexpr int kStride = kNumCvtWarps * 32;
+    constexpr int U = 4;
+    const uint32_t rr = static_cast<uint32_t>(ct) >> cshift;
+    const uint32_t cir = static_cast<uint32_t>(ct) & ((1u << cshift) - 1u);
+    const uint32_t off0 = rr * bkb + 32u * cir;
+    const uint32_t off1 = off0 + 16u;
+    const uint32_t d0 = adst + (off0 ^ (((off0 >> 7) & sw) << 4));
+    const uint32_t d1 = adst + (off1 ^ (((off1 >> 7) & sw) << 4));
+    const uint32_t dstep = (static_cast<uint32_t>(kStride) >> cshift) * bkb;
+    const uint32_t s0 = stg + 16u * static_cast<uint32_t>(ct);
+    int i = 0;
+    const int n_mine = ct < nchunks ? (nchunks - ct + kStride - 1) / kStride : 0;
+    for (; i + U <= n_mine; i += U) {
+        uint4 pk[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) pk[u] = lds128u(s0 + 16u * kStride * static_cast<uint32_t>(i + u));
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            uint32_t o[8];
+            widen_word(pk[u].x, sgn, o[0], o[1]);
+            widen_word(pk[u].y, sgn, o[2], o[3]);
+            widen_word(pk[u].z, sgn, o[4], o[5]);
+            widen_word(pk[u].w, sgn, o[6], o[7]);
+            const uint32_t dd = dstep * static_cast<uint32_t>(i + u);
+            sts128(d0 + dd, o[0], o[1], o[2], o[3]);
+            sts128(d1 + dd, o[4], o[5], o[6], o[7]);
+        }
+    }
+    for (; i < n_mine; ++i) {
+        const uint4 pk = lds128u(s0 + 16u * kStride * static_cast<uint32_t>(i));
+        uint32_t o[8];
+        widen_word(pk.x, sgn, o[0], o[1]);
+        widen_word(pk.y, sgn, o[2], o[3]);
+        widen_word(pk.z, sgn, o[4], o[5]);
+        widen_word(pk.w, sgn, o[6], o[7]);
+        const uint32_t dd = dstep * static_cast<uint32_t>(i);
+        sts128(d0 + dd, o[0], o[1], o[2], o[3]);
+        sts128(d1 + dd, o[4], o[5], o[6], o[7]);
+    }
+}
+
 template <bool IS4, int OUT, bool ZX>
 __global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
 qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap wmap,
@@ -643,29 +707,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 if (ct == 0) trace_ev(p, 8, cstage++);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
-                for (int g = ct; g < nchunks; g += kNumCvtWarps * 32) {
-                    const uint32_t rr = static_cast<uint32_t>(g) >> cshift;
-                    const uint32_t cir = static_cast<uint32_t>(g) & ((1u << cshift) - 1u);
-                    const uint4 pk = lds128u(stg + 16u * static_cast<uint32_t>(g));
-                    const uint32_t src4[4] = {pk.x, pk.y, pk.z, pk.w};
-                    uint32_t o[8];
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        uint32_t lo = src4[j] & 0x0F0F0F0Fu;
-                        uint32_t hi = (src4[j] >> 4) & 0x0F0F0F0Fu;
-                        if (sgn) {
-                            lo = ((lo ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
-                            hi = ((hi ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
-                        }
-                        o[2 * j] = __byte_perm(lo, hi, 0x5140);
-                        o[2 * j + 1] = __byte_perm(lo, hi, 0x7362);
-                    }
-                    // widened bytes [32*cir, 32*cir+32) of row rr, swizzled like the TMA would
-                    const uint32_t off0 = rr * bkb + 32u * cir;
-                    const uint32_t off1 = off0 + 16u;
-                    sts128(adst + (off0 ^ (((off0 >> 7) & sw) << 4)), o[0], o[1], o[2], o[3]);
-                    sts128(adst + (off1 ^ (((off1 >> 7) & sw) << 4)), o[4], o[5], o[6], o[7]);
-                }
+                widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, sgn);
                 fence_proxy_async_smem();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&aready[stage]);

@@ -223,7 +223,6 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         const int ct = (warp - kWarpCvt0) * 32 + lane;
         const bool sgn = ((p.idesc >> 7) & 1u) != 0;
         const int npix = p.HR * p.Wh;
-        const int nchunks = npix * (p.nplanes / 2);
         int g = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
             const int stage = g % NS;
@@ -232,26 +231,39 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             if (ct == 0) trace_ev(p, 8, g);
             const uint32_t src = smem_u32(smem + p.off_hp + stage * p.hp_stage_bytes);
             const uint32_t dst = smem_u32(smem + p.off_hx + stage * p.hx_stage_bytes);
-            for (int c = ct; c < nchunks; c += kNumCvtWarps * 32) {
-                const int j = c / npix;
-                const int px = c - j * npix;
-                const uint4 pk = lds128u(src + static_cast<uint32_t>(c) * 16u);
-                const uint32_t s4[4] = {pk.x, pk.y, pk.z, pk.w};
-                uint32_t o[8];
+            constexpr int kStride = kNumCvtWarps * 32;
+            constexpr int U = 4;            // loads batched ahead of the conversion
+            for (int j = 0; j < p.nplanes / 2; ++j) {
+                const uint32_t sj = src + static_cast<uint32_t>(j * npix) * 16u;
+                const uint32_t dj = dst + static_cast<uint32_t>(2 * j) * p.h_plane_bytes;
+                int px = ct;
+                for (; px + (U - 1) * kStride < npix; px += U * kStride) {
+                    uint4 pk[U];
 #pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                    uint32_t lo = s4[i] & 0x0F0F0F0Fu;
-                    uint32_t hi = (s4[i] >> 4) & 0x0F0F0F0Fu;
-                    if (sgn) {
-                        lo = ((lo ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
-                        hi = ((hi ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
+                    for (int u = 0; u < U; ++u) pk[u] = lds128u(sj + static_cast<uint32_t>(px + u * kStride) * 16u);
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        uint32_t o[8];
+                        widen_word(pk[u].x, sgn, o[0], o[1]);
+                        widen_word(pk[u].y, sgn, o[2], o[3]);
+                        widen_word(pk[u].z, sgn, o[4], o[5]);
+                        widen_word(pk[u].w, sgn, o[6], o[7]);
+                        const uint32_t d0 = dj + static_cast<uint32_t>(px + u * kStride) * 16u;
+                        sts128(d0, o[0], o[1], o[2], o[3]);
+                        sts128(d0 + p.h_plane_bytes, o[4], o[5], o[6], o[7]);
                     }
-                    o[2 * i] = __byte_perm(lo, hi, 0x5140);
-                    o[2 * i + 1] = __byte_perm(lo, hi, 0x7362);
                 }
-                const uint32_t d0 = dst + static_cast<uint32_t>(2 * j) * p.h_plane_bytes + static_cast<uint32_t>(px) * 16u;
-                sts128(d0, o[0], o[1], o[2], o[3]);
-                sts128(d0 + p.h_plane_bytes, o[4], o[5], o[6], o[7]);
+                for (; px < npix; px += kStride) {
+                    const uint4 pk = lds128u(sj + static_cast<uint32_t>(px) * 16u);
+                    uint32_t o[8];
+                    widen_word(pk.x, sgn, o[0], o[1]);
+                    widen_word(pk.y, sgn, o[2], o[3]);
+                    widen_word(pk.z, sgn, o[4], o[5]);
+                    widen_word(pk.w, sgn, o[6], o[7]);
+                    const uint32_t d0 = dj + static_cast<uint32_t>(px) * 16u;
+                    sts128(d0, o[0], o[1], o[2], o[3]);
+                    sts128(d0 + p.h_plane_bytes, o[4], o[5], o[6], o[7]);
+                }
             }
             fence_proxy_async_smem();
             __syncwarp();

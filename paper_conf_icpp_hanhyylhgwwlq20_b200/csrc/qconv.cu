@@ -20,6 +20,7 @@
 #include "conv_fwd.cuh"
 #include "prep.cuh"
 #include "halo.cuh"
+#include "trans.cuh"
 
 namespace {
 
@@ -302,7 +303,7 @@ CUtensorMapSwizzle swizzle_for(int bk) {
 }
 
 qc_status encode_x_map(const qconv_desc *d, const Geometry &g, const void *x, int box_bytes,
-                       CUtensorMapSwizzle sw, CUtensorMap *map) {
+                       CUtensorMapSwizzle sw, CUtensorMap *map, int pixels = qc::kBM) {
     const Driver &drv = driver();
     if (!drv.im2col) return cuda_fail(drv.err);
     const cuuint64_t cb = static_cast<cuuint64_t>(g.c_bytes);
@@ -314,7 +315,7 @@ qc_status encode_x_map(const qconv_desc *d, const Geometry &g, const void *x, in
     cuuint32_t estr[4] = {1, static_cast<cuuint32_t>(d->stride_w), static_cast<cuuint32_t>(d->stride_h), 1};
     CUresult r = drv.im2col(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, const_cast<void *>(x), dims,
                             strides, lower, upper, static_cast<cuuint32_t>(box_bytes),
-                            static_cast<cuuint32_t>(qc::kBM), estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            static_cast<cuuint32_t>(pixels), estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                             sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
     small_tensor_fixup(map, static_cast<uint64_t>(g.x_bytes));
@@ -338,21 +339,51 @@ qc_status encode_w_map(const qconv_desc *d, const Geometry &g, const void *w8, i
     return QC_OK;
 }
 
-qc_status encode_y_map(const qconv_desc *d, const Geometry &g, void *y, int gw, CUtensorMap *map) {
+qc_status encode_y_map(const qconv_desc *d, const Geometry &g, void *y, int gw, CUtensorMap *map,
+                       int rows = qc::kBM, bool swizzle = true) {
     const Driver &drv = driver();
     if (!drv.tiled) return cuda_fail(drv.err);
     const int yb = dtype_bits(d->y_t);
     const cuuint64_t row = static_cast<cuuint64_t>(d->k) * yb / 8;
     cuuint64_t dims[2] = {row, static_cast<cuuint64_t>(g.M)};
     cuuint64_t strides[1] = {row};
-    cuuint32_t box[2] = {static_cast<cuuint32_t>(gw), static_cast<cuuint32_t>(qc::kBM)};
+    cuuint32_t box[2] = {static_cast<cuuint32_t>(gw), static_cast<cuuint32_t>(rows)};
     cuuint32_t estr[2] = {1, 1};
     CUresult r = drv.tiled(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, y, dims, strides, box, estr,
-                           CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_for(gw),
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle ? swizzle_for(gw) : CU_TENSOR_MAP_SWIZZLE_NONE,
                            CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
     small_tensor_fixup(map, static_cast<uint64_t>(g.y_bytes));
     return QC_OK;
+}
+
+// Debug hooks (never set in normal use): QC_EXPERIMENT=<flags> ablations, and
+// QC_TRACE=<file> timestamps of CTA 0's pipeline events, appended to the file after a sync.
+qc::ConvParams debug_params(const qc::ConvParams &base, cudaStream_t stream) {
+    static const char *trace_file = std::getenv("QC_TRACE");
+    static const char *exp_env = std::getenv("QC_EXPERIMENT");
+    qc::ConvParams cp = base;
+    cp.exp_flags = exp_env ? std::atoi(exp_env) : 0;
+    cp.trace = nullptr;
+    if (trace_file) {
+        unsigned long long *tbuf = nullptr;
+        cudaMalloc(&tbuf, 16 * 1024 * sizeof(unsigned long long));
+        cudaMemsetAsync(tbuf, 0, 16 * 1024 * sizeof(unsigned long long), stream);
+        cp.trace = tbuf;
+    }
+    return cp;
+}
+
+void debug_dump(const qc::ConvParams &cp, cudaStream_t stream) {
+    if (!cp.trace) return;
+    std::vector<unsigned long long> h(16 * 1024);
+    cudaMemcpyAsync(h.data(), cp.trace, h.size() * 8, cudaMemcpyDeviceToHost, stream);
+    cudaStreamSynchronize(stream);
+    cudaFree(cp.trace);
+    if (FILE *f = std::fopen(std::getenv("QC_TRACE"), "ab")) {
+        std::fwrite(h.data(), 8, h.size(), f);
+        std::fclose(f);
+    }
 }
 
 template <bool IS4, int OUT, bool ZX>
@@ -374,29 +405,10 @@ qc_status launch_conv_t(const Plan &pl, const CUtensorMap &xm, const CUtensorMap
     cfg.stream = stream;
     cfg.attrs = nullptr;
     cfg.numAttrs = 0;
-    // debug tracing (QC_TRACE=<file>): timestamps of CTA 0's pipeline events, dumped after a sync
-    static const char *trace_file = std::getenv("QC_TRACE");
-    static const char *exp_env = std::getenv("QC_EXPERIMENT");
-    qc::ConvParams cp = pl.cp;
-    cp.exp_flags = exp_env ? std::atoi(exp_env) : 0;
-    unsigned long long *tbuf = nullptr;
-    if (trace_file) {
-        cudaMalloc(&tbuf, 16 * 1024 * sizeof(unsigned long long));
-        cudaMemsetAsync(tbuf, 0, 16 * 1024 * sizeof(unsigned long long), stream);
-        cp.trace = tbuf;
-    }
+    qc::ConvParams cp = debug_params(pl.cp, stream);
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
     if (e != cudaSuccess) return cuda_fail(e);
-    if (tbuf) {
-        std::vector<unsigned long long> h(16 * 1024);
-        cudaMemcpyAsync(h.data(), tbuf, h.size() * 8, cudaMemcpyDeviceToHost, stream);
-        cudaStreamSynchronize(stream);
-        cudaFree(tbuf);
-        if (FILE *f = std::fopen(trace_file, "ab")) {
-            std::fwrite(h.data(), 8, h.size(), f);
-            std::fclose(f);
-        }
-    }
+    debug_dump(cp, stream);
     return QC_OK;
 }
 
@@ -601,6 +613,121 @@ qc_status launch_halo(const Plan &pl, const CUtensorMap &hm, const CUtensorMap &
     return QC_OK;
 }
 
+// ------------------------------------------------------------------ channel-major 1x1 kernel
+bool trans_disabled() {
+    static const bool off = std::getenv("QC_NO_TRANS") != nullptr;
+    return off;
+}
+
+bool make_trans_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
+    if (trans_disabled()) return false;
+    if (d->r != 1 || d->s != 1 || d->x_zero != 0 || d->y_t == QC_S32) return false;
+    if (d->c % 32 || d->k % 64) return false;
+    const bool is4 = g.bits == 4;
+    // With 4-bit activations the 256-pixel operand tile doubles the on-chip widening per
+    // MAC; for deep inputs (C > 512) that outweighs the cheaper epilogue (measured, r1).
+    if (is4 && d->c > 512) return false;
+    const int ybits = dtype_bits(d->y_t);
+    if ((static_cast<int64_t>(d->k) * ybits / 8) % 16) return false;
+    const int BMc = d->k % 128 == 0 ? 128 : 64;
+    const int BNp = 256;
+    const int BK = choose_bk(d->c);
+    const int bkp = is4 ? BK / 2 : BK;
+    const int n_tiles_n = d->k / BMc;
+    const int64_t m_tiles = (g.M + BNp - 1) / BNp;
+    const int64_t num_tiles = m_tiles * n_tiles_n;
+    if (num_tiles > INT32_MAX) return false;
+    const int row_bytes = BMc * ybits / 8;                 // 32 .. 128
+    const uint32_t ystg_one = static_cast<uint32_t>(BNp * row_bytes);
+    const uint32_t a_bytes = static_cast<uint32_t>(BNp * BK);      // activations
+    const uint32_t b_bytes = static_cast<uint32_t>(BMc * BK);      // weights
+    const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(BNp * bkp) : 0u;
+    const uint32_t per_stage = a_bytes + b_bytes + stg_bytes;
+    const uint32_t fixed = 2u * ystg_one + 2048u;
+    if (fixed + 2 * per_stage > 227u * 1024u) return false;
+    int stages = std::min(static_cast<int>((227u * 1024u - fixed) / per_stage), 16);
+    qc::ConvParams &p = pl->cp;
+    std::memset(&p, 0, sizeof(p));
+    p.M = static_cast<int32_t>(g.M);
+    p.P = g.P; p.Q = g.Q; p.PQ = g.P * g.Q; p.K = d->k;
+    p.BN = BMc;                  // channels per tile (UMMA M)
+    p.Wh = BNp;                  // pixels per tile (UMMA N)
+    p.n_tiles_n = n_tiles_n;
+    p.num_tiles = static_cast<int32_t>(num_tiles);
+    p.chunks = d->c / BK;
+    p.num_kb = p.chunks;
+    p.S = 1; p.R = 1; p.H = d->h; p.W = d->w; p.C8 = d->c;
+    p.stride_h = d->stride_h; p.stride_w = d->stride_w; p.pad_h = d->pad_h; p.pad_w = d->pad_w;
+    p.dil_h = p.dil_w = 1;
+    p.BK = BK; p.bkp = bkp; p.stages = stages;
+    p.sw_layout = BK == 128 ? 2 : (BK == 64 ? 4 : 6);
+    p.sw_mask = BK == 128 ? 7 : (BK == 64 ? 3 : 1);
+    p.cvt_shift = bkp >= 64 ? 2 : (bkp >= 32 ? 1 : 0);
+    p.off_a = 0;
+    p.a_stage_bytes = a_bytes;
+    p.off_b = a_bytes * stages;
+    p.b_stage_bytes = b_bytes;
+    p.off_stg = p.off_b + b_bytes * stages;
+    p.stg_stage_bytes = stg_bytes;
+    p.off_ystg = static_cast<uint32_t>(align_up(p.off_stg + stg_bytes * stages, 1024));
+    p.ystg_bytes = ystg_one;
+    p.y_tma = 1;
+    p.y_gw = row_bytes;
+    p.y_gmask = 0;                 // staging unswizzled: a warp's byte stores hit 8 words
+    p.n_ygroups = 1;
+    p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + 2u * ystg_one, 16));
+    p.off_bar = static_cast<uint32_t>(align_up(p.off_par, 8));
+    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 4) * 8 + 16);
+    pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
+    if (pl->smem_bytes > 227u * 1024u) return false;
+    p.idesc = qc::make_idesc_i8(static_cast<uint32_t>(BMc), static_cast<uint32_t>(BNp),
+                                dtype_signed(d->w_t), dtype_signed(d->x_t));
+    pl->tmem_cols = pow2_cols(2 * BNp);
+    p.tmem_cols = pl->tmem_cols;
+    p.y_zero = d->y_zero; p.clamp_lo = d->clamp_lo; p.clamp_hi = d->clamp_hi;
+    p.need_clamp = (d->clamp_lo > dtype_min(d->y_t) || d->clamp_hi < dtype_max(d->y_t)) ? 1 : 0;
+    p.y_row_bytes = static_cast<int64_t>(d->k) * ybits / 8;
+    const int sms = num_sms();
+    int grid = static_cast<int>(std::min<int64_t>(num_tiles, sms / n_tiles_n * n_tiles_n));
+    grid = std::max(grid, 1);
+    pl->grid = grid;
+    pl->threads = is4 ? 512 : 384;
+    pl->BK = BK; pl->bkp = bkp; pl->BN = BMc; pl->n_tiles_n = n_tiles_n;
+    pl->num_tiles = static_cast<int>(num_tiles); pl->stages = stages; pl->chunks = p.chunks;
+    pl->num_kb = p.num_kb;
+    return true;
+}
+
+template <bool IS4, int OUT, bool M64>
+qc_status launch_trans_m(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
+                         const CUtensorMap &ym, cudaStream_t stream) {
+    auto kern = qc::qconv_t_kernel<IS4, OUT, M64>;
+    static int configured = 0;
+    if (!configured) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+        if (e != cudaSuccess) return cuda_fail(e);
+        configured = 1;
+    }
+    cudaLaunchConfig_t cfg;
+    std::memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
+    cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
+    cfg.dynamicSmemBytes = pl.smem_bytes;
+    cfg.stream = stream;
+    qc::ConvParams cp = debug_params(pl.cp, stream);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
+    if (e != cudaSuccess) return cuda_fail(e);
+    debug_dump(cp, stream);
+    return QC_OK;
+}
+
+template <bool IS4, int OUT>
+qc_status launch_trans(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
+                       const CUtensorMap &ym, cudaStream_t stream) {
+    return pl.BN == 64 ? launch_trans_m<IS4, OUT, true>(pl, xm, wm, ym, stream)
+                       : launch_trans_m<IS4, OUT, false>(pl, xm, wm, ym, stream);
+}
+
 }  // namespace
 
 // ====================================================================== C ABI
@@ -781,6 +908,31 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
                 case QC_S8: return is4 ? launch_halo<true, qc::OUT_S8>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_S8>(hp, hm, bm, ym, st);
                 case QC_U4: return is4 ? launch_halo<true, qc::OUT_U4>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_U4>(hp, hm, bm, ym, st);
                 case QC_S4: return is4 ? launch_halo<true, qc::OUT_S4>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_S4>(hp, hm, bm, ym, st);
+                default: break;
+            }
+        }
+    }
+    {   // 1x1 convolutions: channel-major kernel (per-channel constants in registers)
+        Plan tp;
+        if (need_z == 0 && make_trans_plan(d, g, &tp)) {
+            tp.cp.bias = bias;
+            tp.cp.mult = multiplier;
+            tp.cp.shift = shift;
+            tp.cp.y = y;
+            alignas(64) CUtensorMap xm, wm, ym;
+            s = encode_x_map(d, g, x, tp.bkp, g.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(tp.BK), &xm,
+                             tp.cp.Wh);
+            if (s != QC_OK) return s;
+            s = encode_w_map(d, g, w8, tp.BK, tp.BN, swizzle_for(tp.BK), &wm);
+            if (s != QC_OK) return s;
+            s = encode_y_map(d, g, y, tp.cp.y_gw, &ym, tp.cp.Wh, false);
+            if (s != QC_OK) return s;
+            const bool is4 = g.bits == 4;
+            switch (d->y_t) {
+                case QC_U8: return is4 ? launch_trans<true, qc::OUT_U8>(tp, xm, wm, ym, st) : launch_trans<false, qc::OUT_U8>(tp, xm, wm, ym, st);
+                case QC_S8: return is4 ? launch_trans<true, qc::OUT_S8>(tp, xm, wm, ym, st) : launch_trans<false, qc::OUT_S8>(tp, xm, wm, ym, st);
+                case QC_U4: return is4 ? launch_trans<true, qc::OUT_U4>(tp, xm, wm, ym, st) : launch_trans<false, qc::OUT_U4>(tp, xm, wm, ym, st);
+                case QC_S4: return is4 ? launch_trans<true, qc::OUT_S4>(tp, xm, wm, ym, st) : launch_trans<false, qc::OUT_S4>(tp, xm, wm, ym, st);
                 default: break;
             }
         }

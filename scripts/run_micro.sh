@@ -1,3 +1,3 @@
 #!/bin/bash
 mkdir -p gpurun_out
-./scripts/micro/mma_bench > gpurun_out/mma_bench.txt 2>&1
+timeout 120 ./scripts/micro/cvt_bench > gpurun_out/cvt_bench.txt 2>&1

@@ -21,7 +21,7 @@ for name, bits in [(a, int(b)) for a, b in (s.split(':') for s in sys.argv[2:])]
         y = qc.qconv2d_forward(d, x, w, b, mm, nn)
     torch.cuda.synchronize()
 t = np.fromfile(out, dtype=np.uint64).reshape(-1, 16, 1024).astype(np.int64)[-1]
-names = ["prod_empty_ok", "-", "mma_tempty_ok", "mma_full_ok", "mma_commit_tfull", "epi_tfull_ok", "epi_tempty_arrive", "epi_store_issued", "cvt_full_ok", "cvt_done"]
+names = ["prod_empty_ok", "-", "mma_tempty_ok", "mma_full_ok", "mma_commit_tfull", "epi_tfull_ok", "epi_tempty_arrive", "epi_store_issued", "cvt_full_ok", "cvt_done", "cvt_loop_done"]
 t0 = min(v for v in t.reshape(-1) if v > 0)
 for ev, nm in enumerate(names):
     row = t[ev]
