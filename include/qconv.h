@@ -100,9 +100,15 @@ typedef struct {
 /*
  * qconv_prepare_weights -- once-per-layer weight preparation (the paper's
  * "pre-processing"): KRSC weights of dtype d->w_t are widened to the
- * kernel's operand layout, int8 KRSC (4-bit codes sign/zero-extended, since
- * sm_100 tensor cores have no 4-bit integer MMA).  Output bytes:
- * qconv_prepared_weight_bytes(d) = k*r*s*c.  8-bit weights are copied.
+ * kernel's operand layout (sm_100 tensor cores have no 4-bit integer MMA).
+ * 8-bit weights are copied: k*r*s*c bytes.  4-bit weights (c % 32 == 0, else
+ * UNSUPPORTED) become "nibble-plane" int8 KRSC -- within each 32-channel group
+ * of a (k,r,s) row the 16 even channels come first as 16*w, then the 16 odd
+ * channels as w, matching the kernel's on-chip activation widening -- followed,
+ * 16-byte aligned, by int32 wsum[k] = sum over (r,s,c) of w (the correction of
+ * signed 4-bit activations).  The layout is opaque to callers: only
+ * qconv2d_forward (w_prepared = 1) reads it.
+ * qconv_prepared_weight_bytes(d) = k*r*s*c (8-bit) or align16(k*r*s*c) + 4*k.
  *   w       device, packed KRSC (d->w_t)
  *   w_prep  device, >= qconv_prepared_weight_bytes(d) bytes
  * Errors: INVALID_ARG, MISALIGNED, CUDA.
@@ -114,7 +120,7 @@ qc_status qconv_prepare_weights(const qconv_desc *d, const void *w, void *w_prep
  * qconv2d_workspace_size -- device workspace bytes qconv2d_forward needs for
  * this descriptor: 0 unless x_zero != 0 (zero-point border table,
  * k*(r+1)*(s+1) int32) or 4-bit weights are passed unprepared (w_prepared = 0:
- * room for the widened copy).  Returns 0 for an invalid descriptor.
+ * room for the prepared copy, qconv_prepared_weight_bytes(d) rounded up to 256).  Returns 0 for an invalid descriptor.
  */
 size_t qconv2d_workspace_size(const qconv_desc *d);
 

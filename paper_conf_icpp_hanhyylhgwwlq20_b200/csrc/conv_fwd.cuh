@@ -69,6 +69,10 @@ struct ConvParams {
     int32_t y_zero, clamp_lo, clamp_hi, x_zero;
     const int32_t *bias, *mult, *shift;
     const int32_t *zx_table;          // [K][(R+1)*(S+1)] inclusive 2-D prefix sums of sum_c w
+    // 4-bit activations (nibble-plane widening, see widen_word): the accumulator holds
+    // 2^acc_lg * (acc + 8*sum_w if x_sgn4) -- acc_lg = 4 for 4-bit inputs, 0 for 8-bit
+    int32_t acc_lg, x_sgn4;
+    const int32_t *wsum;              // [K] sum_{r,s,c} w (true values) when x_sgn4, else null
     void *y;
     int64_t y_row_bytes;
 };
@@ -170,7 +174,7 @@ __device__ __forceinline__ void epi_general16(const ConvParams &p, uint32_t (&v)
 #pragma unroll
     for (int j = H; j < H + 16; ++j) {
         const int4 pr = lds128(par_addr + 16u * j);
-        int32_t x = static_cast<int32_t>(v[j]) + pr.x;
+        int32_t x = (static_cast<int32_t>(v[j]) >> p.acc_lg) + pr.x;
         if (ZX) {
             const int k = min(kc + j, p.K - 1);
             const int RS1 = p.S + 1;
@@ -308,35 +312,55 @@ __device__ __forceinline__ void epi_half(const ConvParams &p, uint32_t (&v)[32],
 
 // Per-column epilogue constants for the N tile at n0 (see EpiCol); called by all
 // kNumEpiWarps epilogue warps together; thread (ew, lane) owns column 32*ew+lane.
+// Effective bias of column k in units of the true accumulator: the caller's bias, minus
+// 8*sum_w when signed 4-bit activations were widened with the +8 offset (widen_word).
+__device__ __forceinline__ int64_t eff_bias(const ConvParams &p, int k) {
+    int64_t b = p.bias ? __ldg(p.bias + k) : 0;
+    if (p.wsum) b -= 8 * static_cast<int64_t>(__ldg(p.wsum + k));
+    return b;
+}
+
+// Per-column epilogue constants for the N tile at n0 (see EpiCol); called by all
+// kNumEpiWarps epilogue warps together; thread (ew, lane) owns column 32*ew+lane.
+// With acc_lg = L the accumulator is 2^L * (acc + offset): the fast/mid modes use the
+// shift n + L and the bias 2^L * b_eff (the same rational, so the same exactness proofs),
+// which needs |b_eff| < 2^26 (|2^L b_eff| < 2^30, |2^L b_eff m| < 2^61); the general mode
+// shifts the accumulator back first.
 template <int OUT>
 __device__ __forceinline__ void fill_epilogue_params(const ConvParams &p, EpiCol *par, int4 *chunk_info,
                                                      int n0, int ew, int lane, bool force_general) {
     named_bar_sync(1, kNumEpiWarps * 32);
     const int c = ew * 32 + lane;
     const int k = n0 + c;
+    const int lg = p.acc_lg;
+    const int64_t beff = k < p.K ? eff_bias(p, k) : 0;
     EpiCol e;
-    e.b = (p.bias && k < p.K) ? __ldg(p.bias + k) : 0;
+    e.b = static_cast<int32_t>(beff);
     e.m = 0; e.c2 = 0; e.c3 = 0;
-    int32_t nn = 40;
+    int32_t nn = 40 - lg;
     if (OUT != OUT_S32 && k < p.K) {
         e.m = __ldg(p.mult + k);
         nn = __ldg(p.shift + k);
     }
-    const bool all_fast = __ballot_sync(0xffffffffu, nn >= 33 && nn <= 52) == 0xffffffffu;
-    const bool all_mid = __ballot_sync(0xffffffffu, nn >= 20 && nn <= 50) == 0xffffffffu;
+    const int ne = nn + lg;
+    const bool b_ok = lg == 0 ? (beff == static_cast<int64_t>(static_cast<int32_t>(beff)))
+                              : (beff > -(int64_t(1) << 26) && beff < (int64_t(1) << 26));
+    const bool all_fast = __ballot_sync(0xffffffffu, b_ok && ne >= 33 && ne <= 52) == 0xffffffffu;
+    const bool all_mid = __ballot_sync(0xffffffffu, b_ok && ne >= 20 && ne <= 50) == 0xffffffffu;
     const int mode = force_general ? 2 : (all_fast ? 0 : (all_mid ? 1 : 2));
-    const int T = max(33, __reduce_max_sync(0xffffffffu, nn));
+    const int T = max(33, __reduce_max_sync(0xffffffffu, ne));
     if (OUT != OUT_S32 && k < p.K) {
         if (mode == 0) {
-            const int64_t c64 = static_cast<int64_t>(e.b) * e.m + (static_cast<int64_t>(1) << (nn - 1)) +
-                                (static_cast<int64_t>(p.y_zero) << nn);
+            const int64_t c64 = (beff << lg) * e.m + (static_cast<int64_t>(1) << (ne - 1)) +
+                                (static_cast<int64_t>(p.y_zero) << ne);
             e.b = e.m;                                   // {m, sh, C_lo, C_hi}
-            e.m = nn - 32;
+            e.m = ne - 32;
             e.c2 = static_cast<int32_t>(static_cast<uint32_t>(c64));
             e.c3 = static_cast<int32_t>(c64 >> 32);
         } else if (mode == 1) {
-            e.c2 = T - nn;
-            e.c3 = 1 << (nn - 20);
+            e.b = static_cast<int32_t>(beff << lg);
+            e.c2 = T - ne;
+            e.c3 = 1 << (ne - 20);
         } else {
             e.c2 = nn;
         }
@@ -353,19 +377,20 @@ __device__ __forceinline__ void trace_ev(const ConvParams &p, int ev, int seq) {
 }
 
 // ------------------------------------------------------------------ the kernel
-// Widen one 32-bit word of eight packed 4-bit codes (element 2i in the low nibble of byte i)
-// into two words of eight int8 values.  The nibble split uses the FMA pipe (IMAD) where it
-// can, since the integer ALU pipe is half rate and is what bounds the converter warps:
-// lo = w & 0x0F0F0F0F (LOP3), hi = (w - lo) >> 4 (IMAD + IMAD.HI), two byte permutes.
-__device__ __forceinline__ void widen_word(uint32_t w, bool sgn, uint32_t &o0, uint32_t &o1) {
-    uint32_t lo = w & 0x0F0F0F0Fu;
-    uint32_t hi = __umulhi(w - lo, 0x10000000u);
-    if (sgn) {          // sign-extend each nibble: ((v ^ 8) + 0x78) ^ 0x80 per byte
-        lo = ((lo ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
-        hi = ((hi ^ 0x08080808u) + 0x78787878u) ^ 0x80808080u;
-    }
-    o0 = __byte_perm(lo, hi, 0x5140);
-    o1 = __byte_perm(lo, hi, 0x7362);
+// "Nibble-plane" widening of one 32-bit word of eight packed 4-bit codes (element 2i in the
+// low nibble of byte i) into two int8 words with no shifts or byte permutes:
+//   lo = w' & 0x0F0F0F0F  -> bytes = the even elements        (x)
+//   hi = w' & 0xF0F0F0F0  -> bytes = the odd elements times 16 (16 x)
+// where w' = w for unsigned codes and w ^ 0x88888888 for signed ones (x + 8 in [0, 15], so
+// the operand is always unsigned; the OOB zero fill of TMA stays x = 0 after the XOR).
+// The prepared weights compensate (prep.cuh widen_w4_kernel): within every 32-channel
+// group the even channels come first and carry 16 w, the odd channels follow with w, so
+// the MMA sums 16 * x * w over every channel: acc = 16 (acc_true + 8 sum_w [signed]).  The
+// epilogue folds the 16 into the re-quantization shift and the offset into the bias.
+// Two LOP3 per word, versus shift + mask + two PRMT per word for in-order widening.
+__device__ __forceinline__ void widen_word(uint32_t w, uint32_t xo, uint32_t &lo, uint32_t &hi) {
+    lo = (w ^ xo) & 0x0F0F0F0Fu;
+    hi = (w ^ xo) & 0xF0F0F0F0u;
 }
 
 // int4 -> int8 widening of one staged operand tile (Sec.3.2 P:L231-235 bit unpacking,
@@ -375,7 +400,7 @@ __device__ __forceinline__ void widen_word(uint32_t w, bool sgn, uint32_t &o0, u
 // the destination offsets are computed once.  Four chunks are loaded before any is
 // converted so the shared-memory latency overlaps.
 __device__ __forceinline__ void widen_stage(uint32_t stg, uint32_t adst, int ct, int nchunks,
-                                            int cshift, uint32_t bkb, uint32_t sw, bool sgn) {
+                                            int cshift, uint32_t bkb, uint32_t sw, uint32_t xo) {
     constexpr int kStride = kNumCvtWarps * 32;
     constexpr int U = 4;
     const uint32_t rr = static_cast<uint32_t>(ct) >> cshift;
@@ -395,10 +420,10 @@ __device__ __forceinline__ void widen_stage(uint32_t stg, uint32_t adst, int ct,
 #pragma unroll
         for (int u = 0; u < U; ++u) {
             uint32_t o[8];
-            widen_word(pk[u].x, sgn, o[0], o[1]);
-            widen_word(pk[u].y, sgn, o[2], o[3]);
-            widen_word(pk[u].z, sgn, o[4], o[5]);
-            widen_word(pk[u].w, sgn, o[6], o[7]);
+            widen_word(pk[u].x, xo, o[0], o[4]);
+            widen_word(pk[u].y, xo, o[1], o[5]);
+            widen_word(pk[u].z, xo, o[2], o[6]);
+            widen_word(pk[u].w, xo, o[3], o[7]);
             const uint32_t dd = dstep * static_cast<uint32_t>(i + u);
             sts128(d0 + dd, o[0], o[1], o[2], o[3]);
             sts128(d1 + dd, o[4], o[5], o[6], o[7]);
@@ -407,10 +432,10 @@ __device__ __forceinline__ void widen_stage(uint32_t stg, uint32_t adst, int ct,
     for (; i < n_mine; ++i) {
         const uint4 pk = lds128u(s0 + 16u * kStride * static_cast<uint32_t>(i));
         uint32_t o[8];
-        widen_word(pk.x, sgn, o[0], o[1]);
-        widen_word(pk.y, sgn, o[2], o[3]);
-        widen_word(pk.z, sgn, o[4], o[5]);
-        widen_word(pk.w, sgn, o[6], o[7]);
+        widen_word(pk.x, xo, o[0], o[4]);
+        widen_word(pk.y, xo, o[1], o[5]);
+        widen_word(pk.z, xo, o[2], o[6]);
+        widen_word(pk.w, xo, o[3], o[7]);
         const uint32_t dd = dstep * static_cast<uint32_t>(i);
         sts128(d0 + dd, o[0], o[1], o[2], o[3]);
         sts128(d1 + dd, o[4], o[5], o[6], o[7]);
@@ -696,7 +721,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
         int cstage = 0;
         const int cshift = p.cvt_shift;                      // log2(16-byte packed chunks/pixel)
         const int nchunks = kBM << cshift;
-        const bool sgn = ((p.idesc >> 7) & 1u) != 0;
+        const uint32_t xo = p.x_sgn4 ? 0x88888888u : 0u;
         const uint32_t sw = static_cast<uint32_t>(p.sw_mask);
         const uint32_t bkb = static_cast<uint32_t>(p.BK);
         int stage = 0;
@@ -707,7 +732,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 if (ct == 0) trace_ev(p, 8, cstage++);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
-                widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, sgn);
+                widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo);
                 fence_proxy_async_smem();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&aready[stage]);

@@ -221,7 +221,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         // packed plane j (16 B = 32 channels per pixel) -> int8 planes 2j (channels 0..15)
         // and 2j+1 (16..31) at the same pixel offset
         const int ct = (warp - kWarpCvt0) * 32 + lane;
-        const bool sgn = ((p.idesc >> 7) & 1u) != 0;
+        const uint32_t xo = p.x_sgn4 ? 0x88888888u : 0u;
         const int npix = p.HR * p.Wh;
         int g = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
@@ -244,10 +244,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
 #pragma unroll
                     for (int u = 0; u < U; ++u) {
                         uint32_t o[8];
-                        widen_word(pk[u].x, sgn, o[0], o[1]);
-                        widen_word(pk[u].y, sgn, o[2], o[3]);
-                        widen_word(pk[u].z, sgn, o[4], o[5]);
-                        widen_word(pk[u].w, sgn, o[6], o[7]);
+                        widen_word(pk[u].x, xo, o[0], o[4]);
+                        widen_word(pk[u].y, xo, o[1], o[5]);
+                        widen_word(pk[u].z, xo, o[2], o[6]);
+                        widen_word(pk[u].w, xo, o[3], o[7]);
                         const uint32_t d0 = dj + static_cast<uint32_t>(px + u * kStride) * 16u;
                         sts128(d0, o[0], o[1], o[2], o[3]);
                         sts128(d0 + p.h_plane_bytes, o[4], o[5], o[6], o[7]);
@@ -256,10 +256,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 for (; px < npix; px += kStride) {
                     const uint4 pk = lds128u(sj + static_cast<uint32_t>(px) * 16u);
                     uint32_t o[8];
-                    widen_word(pk.x, sgn, o[0], o[1]);
-                    widen_word(pk.y, sgn, o[2], o[3]);
-                    widen_word(pk.z, sgn, o[4], o[5]);
-                    widen_word(pk.w, sgn, o[6], o[7]);
+                    widen_word(pk.x, xo, o[0], o[4]);
+                    widen_word(pk.y, xo, o[1], o[5]);
+                    widen_word(pk.z, xo, o[2], o[6]);
+                    widen_word(pk.w, xo, o[3], o[7]);
                     const uint32_t d0 = dj + static_cast<uint32_t>(px) * 16u;
                     sts128(d0, o[0], o[1], o[2], o[3]);
                     sts128(d0 + p.h_plane_bytes, o[4], o[5], o[6], o[7]);

@@ -1,6 +1,7 @@
 // prep.cuh -- memory-bound kernels around the convolution:
 //   quantize_pack_kernel : fp32/bf16 NHWC -> packed int8/int4 NHWC (Z4)
-//   widen_w4_kernel      : packed int4 KRSC weights -> int8 KRSC (once per layer)
+//   widen_w4_kernel      : packed int4 KRSC weights -> nibble-plane int8 KRSC (once per layer)
+//   wsum_w4_kernel       : per-channel weight sums (signed 4-bit activation offset)
 //   zx_table_kernel      : 2-D prefix sums of sum_c w[k,r,s,c] for x_zero != 0 borders (Z2)
 #pragma once
 #include <cstdint>
@@ -121,20 +122,65 @@ __global__ void __launch_bounds__(256) quantize_pack_kernel(const __grid_constan
     }
 }
 
-// packed int4 -> int8 (sign- or zero-extended); n_bytes_in packed bytes.
+// packed int4 KRSC -> prepared int8 KRSC in the "nibble-plane" order the on-chip activation
+// widening produces (conv_fwd.cuh widen_word): for every 16-byte packed group (32 channels
+// c0..c0+31 of one (k,r,s)), byte p < 16 holds 16 * w[c0 + 2p] and byte 16 + p holds
+// w[c0 + 2p + 1] (sign- or zero-extended; 16 w of a 4-bit code fits 8 bits).  Requires
+// C % 32 == 0.  n_groups = packed bytes / 16.
 __global__ void __launch_bounds__(256) widen_w4_kernel(const uint8_t *__restrict__ w4,
-                                                       int8_t *__restrict__ w8, int64_t n_bytes_in,
+                                                       int8_t *__restrict__ w8, int64_t n_groups,
                                                        int32_t is_signed) {
-    for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n_bytes_in;
+    for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n_groups;
          i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
-        const uint8_t b = w4[i];
-        int lo = b & 0xF, hi = b >> 4;
-        if (is_signed) {
-            lo = lo >= 8 ? lo - 16 : lo;
-            hi = hi >= 8 ? hi - 16 : hi;
+        const uint4 pk = reinterpret_cast<const uint4 *>(w4)[i];
+        const uint32_t wd[4] = {pk.x, pk.y, pk.z, pk.w};
+        uint32_t out[8];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            uint32_t lo = 0, hi = 0;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                int e = (wd[q] >> (8 * j)) & 0xF, o = (wd[q] >> (8 * j + 4)) & 0xF;
+                if (is_signed) {
+                    e = e >= 8 ? e - 16 : e;
+                    o = o >= 8 ? o - 16 : o;
+                }
+                lo |= (static_cast<uint32_t>(16 * e) & 0xFFu) << (8 * j);
+                hi |= (static_cast<uint32_t>(o) & 0xFFu) << (8 * j);
+            }
+            out[q] = lo;
+            out[4 + q] = hi;
         }
-        w8[2 * i] = static_cast<int8_t>(lo);
-        w8[2 * i + 1] = static_cast<int8_t>(hi);
+        uint4 *dst = reinterpret_cast<uint4 *>(w8) + 2 * i;
+        dst[0] = make_uint4(out[0], out[1], out[2], out[3]);
+        dst[1] = make_uint4(out[4], out[5], out[6], out[7]);
+    }
+}
+
+// wsum[k] = sum over (r,s,c) of the true 4-bit weight values of output channel k (row of
+// row_bytes packed bytes): the offset correction of signed 4-bit activations (widen_word).
+__global__ void __launch_bounds__(256) wsum_w4_kernel(const uint8_t *__restrict__ w4,
+                                                      int32_t *__restrict__ wsum, int64_t row_bytes,
+                                                      int32_t is_signed) {
+    const uint8_t *row = w4 + static_cast<int64_t>(blockIdx.x) * row_bytes;
+    int32_t s = 0;
+    for (int64_t i = threadIdx.x; i < row_bytes; i += blockDim.x) {
+        const int b = row[i];
+        int e = b & 0xF, o = b >> 4;
+        if (is_signed) {
+            e = e >= 8 ? e - 16 : e;
+            o = o >= 8 ? o - 16 : o;
+        }
+        s += e + o;
+    }
+    __shared__ int32_t red[8];
+    for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int32_t t = 0;
+        for (int w = 0; w < static_cast<int>(blockDim.x >> 5); ++w) t += red[w];
+        wsum[blockIdx.x] = t;
     }
 }
 
@@ -142,7 +188,7 @@ __global__ void __launch_bounds__(256) widen_w4_kernel(const uint8_t *__restrict
 // For an output pixel whose in-bounds taps are r in [r0,r1), s in [s0,s1) the
 // padded taps' contribution to subtract is x_zero * (T[r1][s1]-T[r0][s1]-T[r1][s0]+T[r0][s0]).
 __global__ void zx_table_kernel(const int8_t *__restrict__ w8, int32_t *__restrict__ table, int K,
-                                int R, int S, int C, int is_unsigned) {
+                                int R, int S, int C, int is_unsigned, int nib) {
     const int k = blockIdx.x * blockDim.x + threadIdx.x;
     if (k >= K) return;
     int32_t *t = table + static_cast<int64_t>(k) * (R + 1) * (S + 1);
@@ -153,8 +199,12 @@ __global__ void zx_table_kernel(const int8_t *__restrict__ w8, int32_t *__restri
         for (int j = 1; j <= S; ++j) {
             const int8_t *src = w8 + ((static_cast<int64_t>(k) * R + (i - 1)) * S + (j - 1)) * C;
             int32_t s = 0;
-            for (int c = 0; c < C; ++c) s += is_unsigned ? static_cast<int32_t>(static_cast<uint8_t>(src[c]))
-                                                         : static_cast<int32_t>(src[c]);
+            for (int c = 0; c < C; ++c) {
+                int32_t v = is_unsigned ? static_cast<int32_t>(static_cast<uint8_t>(src[c]))
+                                        : static_cast<int32_t>(src[c]);
+                if (nib && (c & 31) < 16) v /= 16;       // nibble-plane prepared 4-bit weights
+                s += v;
+            }
             rowsum += s;
             t[i * (S + 1) + j] = t[(i - 1) * (S + 1) + j] + rowsum;
         }

@@ -55,6 +55,9 @@ int64_t dtype_max(qc_dtype t) {
 }
 bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+// MMA operand signedness of the activations: 4-bit codes are widened to unsigned bytes
+// (nibble-plane widening, conv_fwd.cuh widen_word); 8-bit codes are used as they are.
+bool act_signed(const qconv_desc *d) { return dtype_bits(d->x_t) == 8 && dtype_signed(d->x_t); }
 
 // ------------------------------------------------------------------ driver entry points
 typedef CUresult (*PFN_encodeIm2col)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
@@ -181,8 +184,12 @@ qc_status check_supported(const qconv_desc *d, const Geometry &g) {
     const int64_t wmax = std::max(-dtype_min(d->w_t), dtype_max(d->w_t));
     const int64_t xraw = std::max(-dtype_min(d->x_t), dtype_max(d->x_t));
     const int64_t xctr = std::max(d->x_zero - dtype_min(d->x_t), dtype_max(d->x_t) - d->x_zero);
-    const double lim = 2147483647.0;
-    if (static_cast<double>(T) * xraw * wmax > lim || static_cast<double>(T) * xctr * wmax > lim)
+    // 4-bit activations are widened to 16 x (x [+ 8]) (nibble-plane widening): the MMA sum
+    // is 16 x larger and must stay below 2^30 (the epilogue adds 16 * bias inside int32)
+    const double lim = dtype_bits(d->x_t) == 4 ? 67108864.0 /* 2^30 / 16 */ : 2147483647.0;
+    const double xw = dtype_bits(d->x_t) == 4 ? 15.0 : static_cast<double>(std::max(xraw, xctr));
+    if (static_cast<double>(T) * xraw * wmax > lim || static_cast<double>(T) * xctr * wmax > lim ||
+        static_cast<double>(T) * xw * wmax > lim)
         return QC_ERR_OVERFLOW_RISK;
     return QC_OK;
 }
@@ -287,7 +294,7 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.cvt_shift = pl->bkp >= 64 ? 2 : (pl->bkp >= 32 ? 1 : 0);
     p.need_clamp = (d->y_t != QC_S32 && (d->clamp_lo > dtype_min(d->y_t) || d->clamp_hi < dtype_max(d->y_t))) ? 1 : 0;
     p.sw_mask = pl->BK == 128 ? 7 : (pl->BK == 64 ? 3 : 1);
-    p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), dtype_signed(d->x_t), dtype_signed(d->w_t));
+    p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), act_signed(d), dtype_signed(d->w_t));
     p.tmem_cols = pl->tmem_cols;
     p.y_zero = d->y_t == QC_S32 ? 0 : d->y_zero;
     p.clamp_lo = d->y_t == QC_S32 ? INT32_MIN : d->clamp_lo;
@@ -507,7 +514,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 5) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
     if (pl->smem_bytes > 227u * 1024u) return false;
-    p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), dtype_signed(d->x_t), dtype_signed(d->w_t));
+    p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), act_signed(d), dtype_signed(d->w_t));
     pl->tmem_cols = pow2_cols(2 * BN);
     p.tmem_cols = pl->tmem_cols;
     p.y_zero = d->y_zero; p.clamp_lo = d->clamp_lo; p.clamp_hi = d->clamp_hi; p.x_zero = 0;
@@ -681,7 +688,7 @@ bool make_trans_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
     if (pl->smem_bytes > 227u * 1024u) return false;
     p.idesc = qc::make_idesc_i8(static_cast<uint32_t>(BMc), static_cast<uint32_t>(BNp),
-                                dtype_signed(d->w_t), dtype_signed(d->x_t));
+                                dtype_signed(d->w_t), act_signed(d));
     pl->tmem_cols = pow2_cols(2 * BNp);
     p.tmem_cols = pl->tmem_cols;
     p.y_zero = d->y_zero; p.clamp_lo = d->clamp_lo; p.clamp_hi = d->clamp_hi;
@@ -818,10 +825,22 @@ qc_status qconv_quantize_pack(const void *x, qc_ftype xt, int64_t npix, int32_t 
     return QC_OK;
 }
 
+// Prepared weights: int8 KRSC (8-bit: the codes as they are; 4-bit: nibble-plane order,
+// prep.cuh widen_w4_kernel), then for 4-bit a 16-byte aligned int32 wsum[K].
+static size_t prepared_bytes(const qconv_desc *d, const Geometry &g) {
+    if (dtype_bits(d->w_t) == 8) return static_cast<size_t>(g.w8_bytes);
+    return align_up(static_cast<size_t>(g.w8_bytes), 16) + 4 * static_cast<size_t>(d->k);
+}
+static const int32_t *prepared_wsum(const qconv_desc *d, const Geometry &g, const void *w8) {
+    if (dtype_bits(d->w_t) != 4) return nullptr;
+    return reinterpret_cast<const int32_t *>(static_cast<const uint8_t *>(w8) +
+                                             align_up(static_cast<size_t>(g.w8_bytes), 16));
+}
+
 size_t qconv_prepared_weight_bytes(const qconv_desc *d) {
     Geometry g;
     if (validate_desc(d, &g) != QC_OK) return 0;
-    return static_cast<size_t>(g.w8_bytes);
+    return prepared_bytes(d, g);
 }
 
 static qc_status prepare_weights_impl(const qconv_desc *d, const Geometry &g, const void *w,
@@ -832,11 +851,15 @@ static qc_status prepare_weights_impl(const qconv_desc *d, const Geometry &g, co
         if (e != cudaSuccess) return cuda_fail(e);
         return QC_OK;
     }
-    const int64_t nin = g.w8_bytes / 2;
-    const int grid = static_cast<int>(std::min<int64_t>((nin + 255) / 256, 4096));
+    if (d->c % 32) return QC_ERR_UNSUPPORTED;            // nibble planes are 32-channel groups
+    const int64_t ngroups = g.w_bytes / 16;
+    const int grid = static_cast<int>(std::min<int64_t>((ngroups + 255) / 256, 4096));
+    const int sgn = d->w_t == QC_S4 ? 1 : 0;
     qc::widen_w4_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(w),
-                                              static_cast<int8_t *>(w_prep), nin,
-                                              d->w_t == QC_S4 ? 1 : 0);
+                                              static_cast<int8_t *>(w_prep), ngroups, sgn);
+    qc::wsum_w4_kernel<<<d->k, 256, 0, st>>>(
+        static_cast<const uint8_t *>(w), const_cast<int32_t *>(prepared_wsum(d, g, w_prep)),
+        static_cast<int64_t>(d->r) * d->s * d->c / 2, sgn);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e);
     return QC_OK;
@@ -852,7 +875,7 @@ qc_status qconv_prepare_weights(const qconv_desc *d, const void *w, void *w_prep
 }
 
 static size_t ws_weights_bytes(const qconv_desc *d, const Geometry &g) {
-    return (dtype_bits(d->w_t) == 4 && !d->w_prepared) ? align_up(static_cast<size_t>(g.w8_bytes), 256) : 0;
+    return (dtype_bits(d->w_t) == 4 && !d->w_prepared) ? align_up(prepared_bytes(d, g), 256) : 0;
 }
 static size_t ws_zx_bytes(const qconv_desc *d) {
     return d->x_zero != 0 ? align_up(static_cast<size_t>(d->k) * (d->r + 1) * (d->s + 1) * 4, 256) : 0;
@@ -862,6 +885,13 @@ size_t qconv2d_workspace_size(const qconv_desc *d) {
     Geometry g;
     if (validate_desc(d, &g) != QC_OK) return 0;
     return ws_weights_bytes(d, g) + ws_zx_bytes(d);
+}
+
+// Accumulator scale and signed-offset correction of 4-bit activations (widen_word).
+static void set_act_params(const qconv_desc *d, const Geometry &g, const void *w8, qc::ConvParams &p) {
+    p.acc_lg = g.bits == 4 ? 4 : 0;
+    p.x_sgn4 = (g.bits == 4 && d->x_t == QC_S4) ? 1 : 0;
+    p.wsum = p.x_sgn4 ? prepared_wsum(d, g, w8) : nullptr;
 }
 
 qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, const int32_t *bias,
@@ -895,6 +925,7 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
     {   // stride-1 convolutions: halo kernel (one tiled TMA per tile, resident weights)
         Plan hp;
         if (need_z == 0 && make_halo_plan(d, g, &hp)) {
+            set_act_params(d, g, w8, hp.cp);
             hp.cp.bias = bias;
             hp.cp.mult = multiplier;
             hp.cp.shift = shift;
@@ -915,6 +946,7 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
     {   // 1x1 convolutions: channel-major kernel (per-channel constants in registers)
         Plan tp;
         if (need_z == 0 && make_trans_plan(d, g, &tp)) {
+            set_act_params(d, g, w8, tp.cp);
             tp.cp.bias = bias;
             tp.cp.mult = multiplier;
             tp.cp.shift = shift;
@@ -938,10 +970,12 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
         }
     }
     qc::ConvParams &p = pl.cp;
+    set_act_params(d, g, w8, p);
     if (need_z) {
         int32_t *table = reinterpret_cast<int32_t *>(static_cast<uint8_t *>(workspace) + need_w);
         qc::zx_table_kernel<<<(d->k + 127) / 128, 128, 0, st>>>(
-            static_cast<const int8_t *>(w8), table, d->k, d->r, d->s, d->c, dtype_signed(d->w_t) ? 0 : 1);
+            static_cast<const int8_t *>(w8), table, d->k, d->r, d->s, d->c, dtype_signed(d->w_t) ? 0 : 1,
+            g.bits == 4 ? 1 : 0);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return cuda_fail(e);
         p.zx_table = table;

@@ -46,7 +46,7 @@ __device__ __forceinline__ void t_chunk(const ConvParams &p, const TChan &cp, ui
         const int64_t hi64 = static_cast<int64_t>(p.clamp_hi) - p.y_zero;
 #pragma unroll
         for (int j = 0; j < 32; ++j) {
-            const int64_t prod = static_cast<int64_t>(static_cast<int32_t>(v[j]) + cp.b) * cp.m +
+            const int64_t prod = static_cast<int64_t>((static_cast<int32_t>(v[j]) >> p.acc_lg) + cp.b) * cp.m +
                                  (static_cast<int64_t>(1) << (cp.n - 1));
             int64_t t = prod >> cp.n;
             t = t < lo64 ? lo64 : (t > hi64 ? hi64 : t);
@@ -211,22 +211,27 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             if (c0 != cached_c0) {
                 const int k = c0 + ch_local;
                 const bool kok = lane_ok && k < p.K;
-                const int32_t b = (kok && p.bias) ? __ldg(p.bias + k) : 0;
+                const int lg = p.acc_lg;                      // see fill_epilogue_params
+                const int64_t beff = kok ? eff_bias(p, k) : 0;
                 const int32_t m = kok ? __ldg(p.mult + k) : 0;
-                const int32_t n = kok ? __ldg(p.shift + k) : 40;
+                const int32_t n = kok ? __ldg(p.shift + k) : 40 - lg;
+                const int ne = n + lg;
+                const bool b_ok = lg == 0 ? (beff == static_cast<int64_t>(static_cast<int32_t>(beff)))
+                                          : (beff > -(int64_t(1) << 26) && beff < (int64_t(1) << 26));
                 const unsigned act = 0xffffffffu;
-                const bool all_fast = __ballot_sync(act, n >= 33 && n <= 52) == act;
-                const bool all_mid = __ballot_sync(act, n >= 20 && n <= 50) == act;
+                const bool all_fast = __ballot_sync(act, b_ok && ne >= 33 && ne <= 52) == act;
+                const bool all_mid = __ballot_sync(act, b_ok && ne >= 20 && ne <= 50) == act;
                 cp.mode = all_fast ? 0 : (all_mid ? 1 : 2);
-                const int T = max(33, __reduce_max_sync(act, n));
-                cp.m = m; cp.b = b; cp.n = n;
+                const int T = max(33, __reduce_max_sync(act, ne));
+                cp.m = m; cp.b = static_cast<int32_t>(beff); cp.n = n;
                 if (cp.mode == 0) {
-                    cp.c64 = static_cast<int64_t>(b) * m + (static_cast<int64_t>(1) << (n - 1)) +
-                             (static_cast<int64_t>(p.y_zero) << n);
-                    cp.sh = n - 32;
+                    cp.c64 = (beff << lg) * m + (static_cast<int64_t>(1) << (ne - 1)) +
+                             (static_cast<int64_t>(p.y_zero) << ne);
+                    cp.sh = ne - 32;
                 } else if (cp.mode == 1) {
-                    cp.k = T - n;
-                    cp.vlim = 1 << (n - 20);
+                    cp.b = static_cast<int32_t>(beff << lg);
+                    cp.k = T - ne;
+                    cp.vlim = 1 << (ne - 20);
                     cp.sh = T - 32;
                     cp.c64 = static_cast<int64_t>((1 << (T - 33)) + p.y_zero * (1 << (T - 32))) << 32;
                 }
@@ -276,7 +281,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         const int ct = (warp - kWarpCvt0) * 32 + lane;
         const int cshift = p.cvt_shift;
         const int nchunks = BNp << cshift;
-        const bool sgn = ((p.idesc >> 10) & 1u) != 0;     // activations are the B operand here
+        const uint32_t xo = p.x_sgn4 ? 0x88888888u : 0u;
         const uint32_t sw = static_cast<uint32_t>(p.sw_mask);
         const uint32_t bkb = static_cast<uint32_t>(p.BK);
         int g = 0;
@@ -288,7 +293,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 if (ct == 0) trace_ev(p, 8, g);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
-                if (!(p.exp_flags & 8)) widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, sgn);
+                if (!(p.exp_flags & 8)) widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo);
                 if (ct == 0) trace_ev(p, 10, g);
                 fence_proxy_async_smem();
                 __syncwarp();

@@ -13,7 +13,7 @@ __global__ void bench(int reps, int nchunks, int cshift, int bkb, int sw, long l
     __syncthreads();
     long long t0 = clock64();
     for (int r = 0; r < reps; ++r) {
-        widen_stage(stg, adst, threadIdx.x, nchunks, cshift, static_cast<uint32_t>(bkb), static_cast<uint32_t>(sw), false);
+        widen_stage(stg, adst, threadIdx.x, nchunks, cshift, static_cast<uint32_t>(bkb), static_cast<uint32_t>(sw), 0u);
         fence_proxy_async_smem();
         __syncthreads();
     }

@@ -87,10 +87,11 @@ def test_forward_host_validation():
     assert qc.qconv2d_workspace_size(d) == 64 * 16 * 4
     assert _fwd(d) == 5                                                     # WORKSPACE
     d4 = qc.make_desc(**good, x_t=qc.QC_U4, w_t=qc.QC_S4, y_t=qc.QC_U4)
-    assert qc.qconv2d_workspace_size(d4) == 64 * 9 * 64                    # unprepared 4-bit w
+    # prepared 4-bit weights: nibble-plane int8 KRSC + int32 per-channel weight sums
+    assert qc.qconv2d_workspace_size(d4) == 64 * 9 * 64 + 256              # unprepared 4-bit w
     d4.w_prepared = 1
     assert qc.qconv2d_workspace_size(d4) == 0
-    assert qc.qconv_prepared_weight_bytes(d4) == 64 * 9 * 64
+    assert qc.qconv_prepared_weight_bytes(d4) == 64 * 9 * 64 + 4 * 64
 
 
 def test_quantize_host_validation():
