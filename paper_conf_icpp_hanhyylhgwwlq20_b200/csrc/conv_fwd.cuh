@@ -643,7 +643,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                     const int col0 = ci * 32;
                     const uint32_t pa = par_base + 16u * col0;
                     const int4 cinfo = chunk_info[ci];
-                    if (p.exp_flags & 32) {            // experiment: TMEM loads only
+                    if (p.exp_flags & 48) {            // experiment: TMEM loads only
                         uint32_t x = 0;
                         for (int j = 0; j < 32; ++j) x ^= vv[j];
                         if (x == 0x9e3779b9u && col0 == 12345) asm volatile("trap;");

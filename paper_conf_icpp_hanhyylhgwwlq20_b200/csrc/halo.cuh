@@ -90,27 +90,18 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         }
     } else if (warp == kWarpMMA) {
         // ===================== MMA issuer =====================
-        if (lane == 0) {   // one thread issues (measured faster than an elected warp-wide loop)
-            constexpr bool leader = true;
-            // per-MMA descriptor offsets (16-byte units), built once: K order = (r, s, plane pair)
-            uint2 *mtab = reinterpret_cast<uint2 *>(smem + p.off_mtab);
+        {   // the whole warp runs the (uniform) loop, one elected lane issues
+            const bool leader = lane == 0;
+            // per-MMA descriptor offsets (16-byte units) are computed in registers: a table in
+            // shared memory puts a generic load + its latency in front of every MMA issue
             const uint32_t bplane = static_cast<uint32_t>(p.BN) * 16u;
-            {
-                int i = 0;
-                for (int r = 0; r < p.R; ++r)
-                    for (int s = 0; s < p.S; s += (p.tap_pair ? 2 : 1))
-                        for (int j = 0; j < (p.tap_pair ? 1 : p.nplanes); j += 2, ++i) {
-                            const uint32_t aoff = static_cast<uint32_t>(r * p.Wh + s) * 16u +
-                                                  static_cast<uint32_t>(j) * p.h_plane_bytes;
-                            const uint32_t boff = static_cast<uint32_t>(
-                                (p.tap_pair ? (r * p.S + s) : ((r * p.S + s) * p.nplanes + j))) * bplane;
-                            mtab[i] = make_uint2(aoff >> 4, boff >> 4);
-                        }
-            }
-            const int nmma = p.n_mma;
+            const uint32_t a_pl16 = p.h_plane_bytes >> 4, b_pl16 = bplane >> 4;
+            const int sstep = p.tap_pair ? 2 : 1;
+            const int npl = p.tap_pair ? 1 : p.nplanes;
             const uint64_t bdesc0 = make_smem_desc(smem_u32(smem + p.off_bres), bplane, 128u, 0u);
             const uint32_t a_lbo = p.tap_pair ? 16u : p.h_plane_bytes;
             mbar_wait(bfull, 0);
+            __syncwarp();
             tc_fence_after();
             int it = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
@@ -120,19 +111,30 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 const uint32_t phase = static_cast<uint32_t>(it / NS) & 1u;
                 mbar_wait(&tempty[buf], acc_phase ^ 1u);
                 if (leader) trace_ev(p, 2, it);
-                tc_fence_after();
                 mbar_wait(IS4 ? &hready[stage] : &hfull[stage], phase);
                 if (leader) trace_ev(p, 3, it);
+                __syncwarp();
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
                 const uint64_t adesc0 = make_smem_desc(smem_u32(smem + p.off_hx + stage * p.hx_stage_bytes),
                                                        a_lbo, 128u, 0u);
-                for (int i = 0; i < nmma; ++i) {
-                    const uint2 o = mtab[i];
-                    mma_i8(d_tmem, adesc0 + o.x, bdesc0 + o.y, p.idesc, i > 0 ? 1u : 0u);
+                uint32_t acc = 0u;
+                for (int r = 0; r < p.R; ++r) {
+                    for (int s = 0; s < p.S; s += sstep) {
+                        const uint32_t tap = static_cast<uint32_t>(r * p.S + s);
+                        uint64_t ad = adesc0 + static_cast<uint32_t>(r * p.Wh + s);
+                        uint64_t bd = bdesc0 + (p.tap_pair ? tap : tap * static_cast<uint32_t>(p.nplanes)) * b_pl16;
+                        for (int j = 0; j < npl; j += 2) {
+                            if (!(p.exp_flags & 4) || acc == 0u)    // debug ablation: one MMA per tile
+                                mma_i8_warp(d_tmem, ad, bd, p.idesc, acc);
+                            acc = 1u;
+                            ad += 2u * a_pl16;
+                            bd += 2u * b_pl16;
+                        }
+                    }
                 }
-                if (leader) mma_commit(&hempty[stage]);
-                if (leader) mma_commit(&tfull[buf]);
+                mma_commit_warp(&hempty[stage]);
+                mma_commit_warp(&tfull[buf]);
                 if (leader) trace_ev(p, 4, it);
             }
         }
@@ -170,6 +172,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             uint32_t va[32], vb[32];
             auto process = [&](uint32_t (&v)[32], int ci) {
                 const int col0 = ci * 32;
+                if (p.exp_flags & 16) {            // debug ablation: TMEM loads only
+                    if (v[0] == 0x9e3779b9u && col0 == 12345) asm volatile("trap;");
+                    return;
+                }
                 const uint32_t pa = par_base + 16u * col0;
                 const int4 cinfo = chunk_info[ci];
                 epi_requant16<OUT, false, 0>(p, v, pa, cinfo, n0 + col0, 0, 0, 0, 0);

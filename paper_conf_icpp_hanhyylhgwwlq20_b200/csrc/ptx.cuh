@@ -126,6 +126,14 @@ __device__ __forceinline__ void tma_load_3d(void *dst, const void *map, uint64_t
         "l"(map), "r"(smem_u32(bar)), "r"(x), "r"(y), "r"(z)
         : "memory");
 }
+__device__ __forceinline__ void tma_load_4d(void *dst, const void *map, uint64_t *bar, int32_t c0,
+                                            int32_t c1, int32_t c2, int32_t c3) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(smem_u32(dst)),
+        "l"(map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+        : "memory");
+}
 __device__ __forceinline__ void tma_load_5d(void *dst, const void *map, uint64_t *bar, int32_t c0,
                                             int32_t c1, int32_t c2, int32_t c3, int32_t c4) {
     asm volatile(
@@ -160,6 +168,15 @@ __device__ __forceinline__ void bulk_wait() {
 __device__ __forceinline__ void sts128(uint32_t addr, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
     asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d)
                  : "memory");
+}
+// staging stores without a "memory" clobber (so the compiler may interleave them with the
+// re-quantization math); ordering against the later fence + barrier is kept because those
+// are asm volatile statements too
+__device__ __forceinline__ void sts8(uint32_t addr, uint32_t a) {
+    asm volatile("st.shared.u8 [%0], %1;" ::"r"(addr), "r"(a));
+}
+__device__ __forceinline__ void sts16(uint32_t addr, uint32_t a) {
+    asm volatile("st.shared.u16 [%0], %1;" ::"r"(addr), "h"(static_cast<uint16_t>(a)));
 }
 __device__ __forceinline__ void sts64(uint32_t addr, uint32_t a, uint32_t b) {
     asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(addr), "r"(a), "r"(b) : "memory");
@@ -201,6 +218,27 @@ __device__ __forceinline__ void mma_i8(uint32_t d_tmem, uint64_t adesc, uint64_t
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
         : "memory");
 }
+// Warp-collective forms: every lane of the warp executes the call with the same (uniform)
+// operands, one elected lane issues.  Keeping the issuing loop warp-uniform lets the
+// compiler hold descriptors in uniform registers (no per-MMA R2UR / elect branch loop).
+__device__ __forceinline__ void mma_i8_warp(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
+                                            uint32_t idesc, uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p, e;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+        : "memory");
+}
+__device__ __forceinline__ void mma_commit_warp(uint64_t *bar) {
+    asm volatile(
+        "{\n\t.reg .pred e;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(
+            static_cast<uint32_t>(__cvta_generic_to_shared(bar)))
+        : "memory");
+}
 // Arrive on `bar` once all previously issued tcgen05 ops of this thread complete.
 __device__ __forceinline__ void mma_commit(uint64_t *bar) {
     asm volatile(
@@ -227,6 +265,17 @@ __device__ __forceinline__ void tmem_wait_ld_regs(uint32_t (&v)[32]) {
 __device__ __forceinline__ void tmem_ld_32x32b_x32(uint32_t taddr, uint32_t (&v)[32]) {
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, "
+        "%11, %12, %13, %14, %15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, "
+        "%28, %29, %30, %31}, [%32];"
+        : QC_R8(0), QC_R8(8), QC_R8(16), QC_R8(24)
+        : "r"(taddr));
+}
+// 16 lanes x 8 columns per repetition, 8 repetitions (64 columns): thread t gets, for
+// repetition k, v[4k+0..1] = lane (base + t/4), columns 8k + 2(t%4) + {0,1}, and
+// v[4k+2..3] = lane (base + t/4 + 8), same columns (measured, scripts/micro/tmem_layout.cu).
+__device__ __forceinline__ void tmem_ld_16x256b_x8(uint32_t taddr, uint32_t (&v)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.16x256b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, "
         "%11, %12, %13, %14, %15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, "
         "%28, %29, %30, %31}, [%32];"
         : QC_R8(0), QC_R8(8), QC_R8(16), QC_R8(24)

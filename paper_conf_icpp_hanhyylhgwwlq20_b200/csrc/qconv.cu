@@ -346,6 +346,27 @@ qc_status encode_w_map(const qconv_desc *d, const Geometry &g, const void *w8, i
     return QC_OK;
 }
 
+// Weights of the channel-major kernel (trans.cuh): a 4-D view {kg bytes, 8, 2, k/16} with
+// strides {2 kg, kg, 16 kg} so that the tile's shared-memory row r = pl + 8 par + 16 ph holds
+// channel 2 pl + par + 16 ph -- TMEM lanes l and l+8 of every 16-lane group then hold the
+// channel pair (2i, 2i+1).  Requires k % 16 == 0.
+qc_status encode_w_map_pairs(const qconv_desc *d, const Geometry &g, const void *w8, int bk, int bm,
+                             CUtensorMapSwizzle sw, CUtensorMap *map) {
+    const Driver &drv = driver();
+    if (!drv.tiled) return cuda_fail(drv.err);
+    const cuuint64_t kg = static_cast<cuuint64_t>(d->r) * d->s * d->c;
+    cuuint64_t dims[4] = {kg, 8, 2, static_cast<cuuint64_t>(d->k / 16)};
+    cuuint64_t strides[3] = {2 * kg, kg, 16 * kg};
+    cuuint32_t box[4] = {static_cast<cuuint32_t>(bk), 8, 2, static_cast<cuuint32_t>(bm / 16)};
+    cuuint32_t estr[4] = {1, 1, 1, 1};
+    CUresult r = drv.tiled(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, const_cast<void *>(w8), dims,
+                           strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+    small_tensor_fixup(map, static_cast<uint64_t>(g.w8_bytes));
+    return QC_OK;
+}
+
 qc_status encode_y_map(const qconv_desc *d, const Geometry &g, void *y, int gw, CUtensorMap *map,
                        int rows = qc::kBM, bool swizzle = true) {
     const Driver &drv = driver();
@@ -597,26 +618,10 @@ qc_status launch_halo(const Plan &pl, const CUtensorMap &hm, const CUtensorMap &
     cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
     cfg.dynamicSmemBytes = pl.smem_bytes;
     cfg.stream = stream;
-    static const char *trace_file = std::getenv("QC_TRACE");
-    qc::ConvParams cp = pl.cp;
-    unsigned long long *tbuf = nullptr;
-    if (trace_file) {
-        cudaMalloc(&tbuf, 16 * 1024 * sizeof(unsigned long long));
-        cudaMemsetAsync(tbuf, 0, 16 * 1024 * sizeof(unsigned long long), stream);
-        cp.trace = tbuf;
-    }
+    qc::ConvParams cp = debug_params(pl.cp, stream);
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, hm, bm, ym, cp);
     if (e != cudaSuccess) return cuda_fail(e);
-    if (tbuf) {
-        std::vector<unsigned long long> h(16 * 1024);
-        cudaMemcpyAsync(h.data(), tbuf, h.size() * 8, cudaMemcpyDeviceToHost, stream);
-        cudaStreamSynchronize(stream);
-        cudaFree(tbuf);
-        if (FILE *f = std::fopen(trace_file, "ab")) {
-            std::fwrite(h.data(), 8, h.size(), f);
-            std::fclose(f);
-        }
-    }
+    debug_dump(cp, stream);
     return QC_OK;
 }
 
@@ -680,7 +685,7 @@ bool make_trans_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.ystg_bytes = ystg_one;
     p.y_tma = 1;
     p.y_gw = row_bytes;
-    p.y_gmask = 0;                 // staging unswizzled: a warp's byte stores hit 8 words
+    p.y_gmask = row_bytes >= 128 ? 7 : (row_bytes == 64 ? 3 : 1);   // staging swizzled like the TMA store
     p.n_ygroups = 1;
     p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + 2u * ystg_one, 16));
     p.off_bar = static_cast<uint32_t>(align_up(p.off_par, 8));
@@ -955,9 +960,9 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
             s = encode_x_map(d, g, x, tp.bkp, g.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(tp.BK), &xm,
                              tp.cp.Wh);
             if (s != QC_OK) return s;
-            s = encode_w_map(d, g, w8, tp.BK, tp.BN, swizzle_for(tp.BK), &wm);
+            s = encode_w_map_pairs(d, g, w8, tp.BK, tp.BN, swizzle_for(tp.BK), &wm);
             if (s != QC_OK) return s;
-            s = encode_y_map(d, g, y, tp.cp.y_gw, &ym, tp.cp.Wh, false);
+            s = encode_y_map(d, g, y, tp.cp.y_gw, &ym, tp.cp.Wh, true);
             if (s != QC_OK) return s;
             const bool is4 = g.bits == 4;
             switch (d->y_t) {

@@ -4,11 +4,14 @@
 // Same method (Alg.2, epilogue P:L223/P:L253/P:L265), operands swapped:
 // the UMMA computes D^T = W * X^T with M = BMc output channels (weights as the A
 // operand) and N = BNp output pixels (im2col activations as the B operand).  A TMEM
-// lane is then one output channel, so each epilogue thread keeps its channel's
-// re-quantization constants in registers (no per-element shared-memory loads): per
-// output one IMAD.HI (with the 64-bit bias/rounding addend), one shift and one
-// saturating pack.  The byte-per-channel results of 32 lanes form 32 contiguous
-// bytes of an NHWC row, staged in shared memory and written by TMA stores.
+// lane is then one output channel.  The weight rows are loaded permuted (a 4-D TMA view,
+// qconv.cu encode_w_map_pairs) so that TMEM lanes l and l+8 of every 16-lane group hold
+// the channel pair (2i, 2i+1); a 16x256b TMEM load then gives each epilogue thread both
+// channels of a pair for two adjacent pixels.  The thread keeps the pair's
+// re-quantization constants in registers (no per-element shared-memory loads) and per
+// output pair does two IMAD.HI (with the 64-bit bias/rounding addend), two shifts and one
+// saturating pack into the pair's byte (4-bit) or 16-bit word (8-bit) of an NHWC row,
+// staged (swizzled) in shared memory and written by TMA stores.
 #pragma once
 #include "conv_fwd.cuh"
 
@@ -16,69 +19,102 @@ namespace qc {
 
 struct TChan {          // per-channel constants held in registers by the epilogue thread
     int64_t c64;        // fast/mid: 64-bit addend of the IMAD.HI (bias*m, rounding, zero point)
-    int32_t m, sh, b, k, vlim, n, mode;
+    int32_t m, sh, b, k, vlim, n;
 };
 
-// Re-quantize one 32-pixel chunk of this thread's channel (Eq.(3)-(4)) and
-// store its bytes into the staging rows (row = pixel, stride ROWB bytes).  `mode` is warp
-// uniform: 0 fast (shift 33..52), 1 mid (shift 20..50), 2 general.
-template <int OUT, int ROWB>
-__device__ __forceinline__ void t_chunk(const ConvParams &p, const TChan &cp, uint32_t (&v)[32],
-                                        uint32_t ystg, int lane, bool lane_ok) {
-    constexpr bool kInt4 = (OUT == OUT_U4 || OUT == OUT_S4);
-    int32_t *y = reinterpret_cast<int32_t *>(v);
-    if (cp.mode == 0) {
-#pragma unroll
-        for (int j = 0; j < 32; ++j) {
-            const int64_t prod = static_cast<int64_t>(static_cast<int32_t>(v[j])) * cp.m + cp.c64;
-            y[j] = static_cast<int32_t>(prod >> 32) >> cp.sh;
-        }
-    } else if (cp.mode == 1) {
-#pragma unroll
-        for (int j = 0; j < 32; ++j) {
-            int32_t x = static_cast<int32_t>(v[j]) + cp.b;
-            x = min(cp.vlim, max(-cp.vlim, x)) << cp.k;
-            const int64_t prod = static_cast<int64_t>(x) * cp.m + cp.c64;
-            y[j] = static_cast<int32_t>(prod >> 32) >> cp.sh;
-        }
+// Re-quantize one accumulator of one channel (Eq.(3)-(4)); `mode` is warp
+// uniform: 0 fast (shift 33..52), 1 mid (shift 20..50), 2 general (see conv_fwd.cuh EpiCol).
+template <int MODE>
+__device__ __forceinline__ int32_t t_requant(const ConvParams &p, const TChan &c, uint32_t acc) {
+    int32_t y;
+    if (MODE == 0) {
+        y = static_cast<int32_t>((static_cast<int64_t>(static_cast<int32_t>(acc)) * c.m + c.c64) >> 32) >> c.sh;
+    } else if (MODE == 1) {
+        int32_t x = static_cast<int32_t>(acc) + c.b;
+        x = min(c.vlim, max(-c.vlim, x)) << c.k;
+        y = static_cast<int32_t>((static_cast<int64_t>(x) * c.m + c.c64) >> 32) >> c.sh;
     } else {
         const int64_t lo64 = static_cast<int64_t>(p.clamp_lo) - p.y_zero;
         const int64_t hi64 = static_cast<int64_t>(p.clamp_hi) - p.y_zero;
+        const int64_t prod = static_cast<int64_t>((static_cast<int32_t>(acc) >> p.acc_lg) + c.b) * c.m +
+                             (static_cast<int64_t>(1) << (c.n - 1));
+        int64_t t = prod >> c.n;
+        t = t < lo64 ? lo64 : (t > hi64 ? hi64 : t);
+        y = static_cast<int32_t>(t) + p.y_zero;
+    }
+    return y;
+}
+
+// 64 pixels (columns) of one channel pair: v from tmem_ld_16x256b_x8, repetition k holds
+// pixels px0 = 8k + 2(lane%4) and px0 + 1 for the even (v[4k], v[4k+1]) and odd
+// (v[4k+2], v[4k+3]) channel.  Stores the pair's byte (4-bit) / 16-bit word (8-bit) of each
+// pixel into the swizzled staging rows.  The swizzle term of row px0 + 8k does not depend on
+// k (rows step by 8, the XOR uses row bits below 8 rows), so the two store addresses are
+// computed once and the repetitions use immediate offsets.
+template <int OUT, int MODE, bool CLAMP, int RB, int GMASK>
+__device__ __forceinline__ void t_pairs(const ConvParams &p, const TChan &ce, const TChan &co,
+                                        const uint32_t (&v)[32], uint32_t ystg, int row0, uint32_t boff) {
+    constexpr bool kInt4 = (OUT == OUT_U4 || OUT == OUT_S4);
+    const uint32_t off0 = static_cast<uint32_t>(row0) * RB + boff, off1 = off0 + RB;
+    const uint32_t a0 = ystg + (off0 ^ (((off0 >> 7) & GMASK) << 4));
+    const uint32_t a1 = ystg + (off1 ^ (((off1 >> 7) & GMASK) << 4));
+    const int32_t lo = p.clamp_lo, hi = p.clamp_hi;
 #pragma unroll
-        for (int j = 0; j < 32; ++j) {
-            const int64_t prod = static_cast<int64_t>((static_cast<int32_t>(v[j]) >> p.acc_lg) + cp.b) * cp.m +
-                                 (static_cast<int64_t>(1) << (cp.n - 1));
-            int64_t t = prod >> cp.n;
-            t = t < lo64 ? lo64 : (t > hi64 ? hi64 : t);
-            y[j] = static_cast<int32_t>(t) + p.y_zero;
+    for (int k = 0; k < 8; ++k) {
+        int32_t ye0 = t_requant<MODE>(p, ce, v[4 * k]), ye1 = t_requant<MODE>(p, ce, v[4 * k + 1]);
+        int32_t yo0 = t_requant<MODE>(p, co, v[4 * k + 2]), yo1 = t_requant<MODE>(p, co, v[4 * k + 3]);
+        if (CLAMP) {
+            ye0 = min(hi, max(lo, ye0)); ye1 = min(hi, max(lo, ye1));
+            yo0 = min(hi, max(lo, yo0)); yo1 = min(hi, max(lo, yo1));
         }
+        const uint32_t d = static_cast<uint32_t>(8 * k * RB);
+        if (kInt4) {
+            sts8(a0 + d, OUT == OUT_U4 ? pack_sat_u4(yo0, ye0, 0u) : pack_sat_s4(yo0, ye0, 0u));
+            sts8(a1 + d, OUT == OUT_U4 ? pack_sat_u4(yo1, ye1, 0u) : pack_sat_s4(yo1, ye1, 0u));
+        } else {
+            sts16(a0 + d, OUT == OUT_U8 ? pack_sat_u8(yo0, ye0, 0u) : pack_sat_s8(yo0, ye0, 0u));
+            sts16(a1 + d, OUT == OUT_U8 ? pack_sat_u8(yo1, ye1, 0u) : pack_sat_s8(yo1, ye1, 0u));
+        }
+    }
+}
+
+template <int OUT, int RB, int GMASK>
+__device__ __forceinline__ void t_pairs_mode(const ConvParams &p, int mode, const TChan &ce, const TChan &co,
+                                             const uint32_t (&v)[32], uint32_t ystg, int row0, uint32_t boff) {
+    if (p.exp_flags & 16) {                       // debug ablation: TMEM loads only
+        if (v[0] == 0x9e3779b9u && row0 == 12345) asm volatile("trap;");
+        return;
     }
     if (p.need_clamp) {
-#pragma unroll
-        for (int j = 0; j < 32; ++j) y[j] = min(p.clamp_hi, max(p.clamp_lo, y[j]));
-    }
-    if (kInt4) {
-        // channel pair (2i, 2i+1) shares a byte: the even lane writes pixels 0..15 of the
-        // chunk, the odd lane pixels 16..31, each fetching its partner's half
-        const bool odd = lane & 1;
-        const uint32_t base = ystg + (odd ? 16u * ROWB : 0u);
-#pragma unroll
-        for (int j = 0; j < 16; ++j) {
-            const int32_t mine = odd ? y[j + 16] : y[j];
-            const int32_t give = odd ? y[j] : y[j + 16];
-            const int32_t other = __shfl_xor_sync(0xffffffffu, give, 1);
-            const int32_t lo = odd ? other : mine;
-            const int32_t hi = odd ? mine : other;
-            const uint32_t byte = OUT == OUT_U4 ? pack_sat_u4(hi, lo, 0u) : pack_sat_s4(hi, lo, 0u);
-            if (lane_ok) asm volatile("st.shared.u8 [%0], %1;" ::"r"(base + j * ROWB), "r"(byte));
-        }
+        if (mode == 0) t_pairs<OUT, 0, true, RB, GMASK>(p, ce, co, v, ystg, row0, boff);
+        else if (mode == 1) t_pairs<OUT, 1, true, RB, GMASK>(p, ce, co, v, ystg, row0, boff);
+        else t_pairs<OUT, 2, true, RB, GMASK>(p, ce, co, v, ystg, row0, boff);
     } else {
-#pragma unroll
-        for (int j = 0; j < 32; ++j) {
-            const uint32_t byte = OUT == OUT_U8 ? pack_sat_u8(0, y[j], 0u) : pack_sat_s8(0, y[j], 0u);
-            if (lane_ok) asm volatile("st.shared.u8 [%0], %1;" ::"r"(ystg + j * ROWB), "r"(byte));
-        }
+        if (mode == 0) t_pairs<OUT, 0, false, RB, GMASK>(p, ce, co, v, ystg, row0, boff);
+        else if (mode == 1) t_pairs<OUT, 1, false, RB, GMASK>(p, ce, co, v, ystg, row0, boff);
+        else t_pairs<OUT, 2, false, RB, GMASK>(p, ce, co, v, ystg, row0, boff);
     }
+}
+
+// Per-channel constants of tile-relative channel k (fill_epilogue_params' rules).
+__device__ __forceinline__ void t_chan_params(const ConvParams &p, int k, bool kok, TChan &c, int &ne, bool &b_ok) {
+    const int lg = p.acc_lg;
+    const int64_t beff = kok ? eff_bias(p, k) : 0;
+    c.m = kok ? __ldg(p.mult + k) : 0;
+    c.n = kok ? __ldg(p.shift + k) : 40 - lg;
+    ne = c.n + lg;
+    b_ok = lg == 0 ? (beff == static_cast<int64_t>(static_cast<int32_t>(beff)))
+                   : (beff > -(int64_t(1) << 26) && beff < (int64_t(1) << 26));
+    c.b = static_cast<int32_t>(beff);
+    c.c64 = (beff << lg) * c.m + (static_cast<int64_t>(1) << (ne - 1)) + (static_cast<int64_t>(p.y_zero) << ne);
+    c.sh = ne - 32;
+}
+__device__ __forceinline__ void t_chan_mid(const ConvParams &p, TChan &c, int ne, int T) {
+    c.b = static_cast<int32_t>(static_cast<int64_t>(c.b) << p.acc_lg);
+    c.k = T - ne;
+    c.vlim = 1 << (ne - 20);
+    c.sh = T - 32;
+    c.c64 = static_cast<int64_t>((1 << (T - 33)) + p.y_zero * (1 << (T - 32))) << 32;
 }
 
 template <bool IS4, int OUT, bool M64>
@@ -96,7 +132,6 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
     constexpr int BNp = kBNp;
     constexpr bool kInt4 = (OUT == OUT_U4 || OUT == OUT_S4);
     constexpr int kRowBytes = BMc * (kInt4 ? 4 : 8) / 8;      // staging row = one pixel
-    constexpr int kChunksPerWarp = kBNp / 32 / 2;             // two warps per lane quarter
 
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem + p.off_bar);
     uint64_t *full = bars;
@@ -153,7 +188,8 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                     uint8_t *xdst = IS4 ? smem + p.off_stg + stage * p.stg_stage_bytes
                                         : smem + p.off_a + stage * p.a_stage_bytes;
                     tma_load_im2col_4d(xdst, &xmap, &full[stage], kb * p.bkp, wb, hb, img, 0, 0);
-                    tma_load_2d(smem + p.off_b + stage * p.b_stage_bytes, &wmap, &full[stage], kb * p.BK, c0);
+                    tma_load_4d(smem + p.off_b + stage * p.b_stage_bytes, &wmap, &full[stage], kb * p.BK, 0, 0,
+                                c0 / 16);
                 }
             }
         }
@@ -191,17 +227,25 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             }
         }
     } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kNumEpiWarps) {
-        // ===================== epilogue: lane = output channel =====================
+        // ===================== epilogue: lane = output channel, thread = channel pair ===========
         const int ew = warp - kWarpEpi0;
         const int quarter = warp & 3;
         const int half = ew >> 2;
-        // M=128: channel = 32*quarter + lane.  M=64 (1-CTA): rows live in lanes 0..15 of
-        // each 32-lane quarter, channel = 16*quarter + lane.
-        const int ch_local = M64 ? 16 * quarter + lane : 32 * quarter + lane;
-        const bool lane_ok = !M64 || lane < 16;
+        // 16-lane group of this warp and its pixel range.  M=128: quarter q holds groups 2q, 2q+1
+        // (one per warp), all 256 pixels.  M=64 (1-CTA): rows live in lanes 0..15 of each quarter
+        // (group q), the two warps of a quarter split the pixels.
+        const int grp = M64 ? quarter : 2 * quarter + half;
+        const uint32_t lane_base = M64 ? 32u * static_cast<uint32_t>(quarter)
+                                       : 32u * static_cast<uint32_t>(quarter) + 16u * static_cast<uint32_t>(half);
+        constexpr int kCols = M64 ? kBNp / 2 : kBNp;
+        const int col_begin = M64 ? half * kCols : 0;
+        const int pair = 8 * grp + (lane >> 2);             // channel pair of the tile
+        constexpr int kGMask = kRowBytes >= 128 ? 7 : (kRowBytes == 64 ? 3 : 1);
+        const uint32_t boff = static_cast<uint32_t>(kInt4 ? pair : 2 * pair);
         const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
         int cached_c0 = -1;
-        TChan cp{};
+        TChan ce{}, co{};
+        int mode = 2;
         int it = 0;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
             const int buf = it & 1;
@@ -209,59 +253,43 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             const int m0 = (tile / p.n_tiles_n) * kBNp;
             const int c0 = (tile % p.n_tiles_n) * BMc;
             if (c0 != cached_c0) {
-                const int k = c0 + ch_local;
-                const bool kok = lane_ok && k < p.K;
-                const int lg = p.acc_lg;                      // see fill_epilogue_params
-                const int64_t beff = kok ? eff_bias(p, k) : 0;
-                const int32_t m = kok ? __ldg(p.mult + k) : 0;
-                const int32_t n = kok ? __ldg(p.shift + k) : 40 - lg;
-                const int ne = n + lg;
-                const bool b_ok = lg == 0 ? (beff == static_cast<int64_t>(static_cast<int32_t>(beff)))
-                                          : (beff > -(int64_t(1) << 26) && beff < (int64_t(1) << 26));
+                const int ke = c0 + 2 * pair, ko = ke + 1;
+                int nee, neo;
+                bool be, bo;
+                t_chan_params(p, ke, ke < p.K, ce, nee, be);
+                t_chan_params(p, ko, ko < p.K, co, neo, bo);
                 const unsigned act = 0xffffffffu;
-                const bool all_fast = __ballot_sync(act, b_ok && ne >= 33 && ne <= 52) == act;
-                const bool all_mid = __ballot_sync(act, b_ok && ne >= 20 && ne <= 50) == act;
-                cp.mode = all_fast ? 0 : (all_mid ? 1 : 2);
-                const int T = max(33, __reduce_max_sync(act, ne));
-                cp.m = m; cp.b = static_cast<int32_t>(beff); cp.n = n;
-                if (cp.mode == 0) {
-                    cp.c64 = (beff << lg) * m + (static_cast<int64_t>(1) << (ne - 1)) +
-                             (static_cast<int64_t>(p.y_zero) << ne);
-                    cp.sh = ne - 32;
-                } else if (cp.mode == 1) {
-                    cp.b = static_cast<int32_t>(beff << lg);
-                    cp.k = T - ne;
-                    cp.vlim = 1 << (ne - 20);
-                    cp.sh = T - 32;
-                    cp.c64 = static_cast<int64_t>((1 << (T - 33)) + p.y_zero * (1 << (T - 32))) << 32;
+                const bool all_fast = __ballot_sync(act, be && bo && nee >= 33 && nee <= 52 && neo >= 33 && neo <= 52) == act;
+                const bool all_mid = __ballot_sync(act, be && bo && nee >= 20 && nee <= 50 && neo >= 20 && neo <= 50) == act;
+                mode = all_fast ? 0 : (all_mid ? 1 : 2);
+                if (mode == 1) {
+                    const int T = max(33, __reduce_max_sync(act, max(nee, neo)));
+                    t_chan_mid(p, ce, nee, T);
+                    t_chan_mid(p, co, neo, T);
                 }
                 cached_c0 = c0;
             }
             mbar_wait(&tfull[buf], acc_phase);
             tc_fence_after();
             if (ew == 0 && lane == 0) trace_ev(p, 5, it);
-            const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
-                                   static_cast<uint32_t>(buf * kBNp);
+            const uint32_t taddr = tmem_base + (lane_base << 16) + static_cast<uint32_t>(buf * kBNp + col_begin);
             const bool storer = ew == 0 && lane == 0;
             if (storer) bulk_wait_read<1>();
             named_bar_sync(1, kNumEpiWarps * 32);
-            // byte of this channel inside a staging row (row = pixel, unswizzled)
-            const uint32_t ystg = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes +
-                                  static_cast<uint32_t>(kInt4 ? ch_local >> 1 : ch_local);
-            // chunks half, half+2, ...: TMEM loads double-buffered against the requantization
+            const uint32_t ystg = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes;
+            const int row0 = col_begin + 2 * (lane & 3);
+            // 64-pixel chunks, TMEM loads double-buffered against the requantization
             uint32_t va[32], vb[32];
-            tmem_ld_32x32b_x32(taddr + half * 32, va);
+            tmem_ld_16x256b_x8(taddr, va);
 #pragma unroll
-            for (int t = 0; t < kChunksPerWarp; t += 2) {
-                const int ci = half + 2 * t;
+            for (int t = 0; t < kCols / 64; t += 2) {
                 tmem_wait_ld_regs(va);
-                if (t + 1 < kChunksPerWarp) tmem_ld_32x32b_x32(taddr + (ci + 2) * 32, vb);
-                t_chunk<OUT, kRowBytes>(p, cp, va, ystg + static_cast<uint32_t>(ci * 32 * kRowBytes), lane, lane_ok);
-                if (t + 1 < kChunksPerWarp) {
+                if (t + 1 < kCols / 64) tmem_ld_16x256b_x8(taddr + static_cast<uint32_t>((t + 1) * 64), vb);
+                t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, va, ystg, row0 + 64 * t, boff);
+                if (t + 1 < kCols / 64) {
                     tmem_wait_ld_regs(vb);
-                    if (t + 2 < kChunksPerWarp) tmem_ld_32x32b_x32(taddr + (ci + 4) * 32, va);
-                    t_chunk<OUT, kRowBytes>(p, cp, vb, ystg + static_cast<uint32_t>((ci + 2) * 32 * kRowBytes), lane,
-                                            lane_ok);
+                    if (t + 2 < kCols / 64) tmem_ld_16x256b_x8(taddr + static_cast<uint32_t>((t + 2) * 64), va);
+                    t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, vb, ystg, row0 + 64 * (t + 1), boff);
                 }
             }
             tc_fence_before();
