@@ -61,6 +61,9 @@ struct ConvParams {
     int32_t Wh, Rt, HR, tiles_per_img, nplanes, nk_planes, tap_pair;
     uint32_t h_plane_bytes, off_hx, off_hp, hx_stage_bytes, hp_stage_bytes, off_bres, b_res_bytes;
     uint32_t halo_tx;
+    int32_t halo_flat;                // halo loaded as whole pixel rows (3-D int64 view): staged
+                                      // pixel-major [HR][Wh][c_px bytes] instead of 16-byte planes
+    int32_t c_px;                     // packed bytes per input pixel (halo_flat)
     uint32_t off_mtab; int32_t n_mma;  // halo: per-MMA descriptor offsets {a>>4, b>>4}
     // shared memory carve-up (byte offsets from the 1024-aligned base)
     uint32_t off_a, off_b, off_stg, off_bar, off_par;
@@ -547,9 +550,12 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
             }
         }
     } else if (warp == kWarpMMA) {
-        // ===================== MMA issuer (one thread) =====================
-        if (lane == 0) {   // one thread issues (measured faster than an elected warp-wide loop)
-            constexpr bool leader = true;
+        // ===================== MMA issuer (whole warp, one elected lane issues) =============
+        // Warp-uniform issue (measured, scripts/micro/commit_bench.cu): ~72 cycles per
+        // 128xNx32 MMA and a free per-stage commit at N=256, versus ~150 cycles per MMA for a
+        // lane-0-only loop.
+        {
+            const bool leader = lane == 0;
             int stage = 0;
             uint32_t phase = 0;
             int it = 0;
@@ -561,12 +567,14 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
                 mbar_wait(&tempty[buf], acc_phase ^ 1u);
                 if (leader) trace_ev(p, 2, it);
+                __syncwarp();
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
                 for (int kb = 0; kb < p.num_kb; ++kb) {
                     mbar_wait(IS4 ? &aready[stage] : &full[stage], phase);
                     if (leader) trace_ev(p, 3, gstage);
                     ++gstage;
+                    __syncwarp();
                     tc_fence_after();
                     const uint32_t a_addr = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
                     const uint32_t b_addr = smem_u32(smem + p.off_b + stage * p.b_stage_bytes);
@@ -575,19 +583,19 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                         // 16-byte K halves (filter taps) are LBO apart, 8-row groups SBO = 128 B
                         const uint64_t ad = make_smem_desc(a_addr, kBM * 16u, 128u, 0u);
                         const uint64_t bd = make_smem_desc(b_addr, static_cast<uint32_t>(p.BN) * 16u, 128u, 0u);
-                        if (leader) mma_i8(d_tmem, ad, bd, p.idesc, kb != 0 ? 1u : 0u);
+                        mma_i8_warp(d_tmem, ad, bd, p.idesc, kb != 0 ? 1u : 0u);
                     } else {
+                        const uint64_t ad0 = make_smem_desc(a_addr, 16u, sbo, p.sw_layout);
+                        const uint64_t bd0 = make_smem_desc(b_addr, 16u, sbo, p.sw_layout);
                         for (int k = 0; k < ksteps; ++k) {
-                            const uint64_t ad = make_smem_desc(a_addr + 32u * k, 16u, sbo, p.sw_layout);
-                            const uint64_t bd = make_smem_desc(b_addr + 32u * k, 16u, sbo, p.sw_layout);
                             if (!(p.exp_flags & 4) || (kb | k) == 0)
-                                if (leader) mma_i8(d_tmem, ad, bd, p.idesc, (kb | k) != 0 ? 1u : 0u);
+                                mma_i8_warp(d_tmem, ad0 + 2u * k, bd0 + 2u * k, p.idesc, (kb | k) != 0 ? 1u : 0u);
                         }
                     }
-                    if (leader) mma_commit(&empty[stage]);
+                    mma_commit_warp(&empty[stage]);
                     if (++stage == NS) { stage = 0; phase ^= 1u; }
                 }
-                if (leader) mma_commit(&tfull[buf]);
+                mma_commit_warp(&tfull[buf]);
                 if (leader) trace_ev(p, 4, it);
             }
         }

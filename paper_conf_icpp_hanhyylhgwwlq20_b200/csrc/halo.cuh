@@ -85,7 +85,11 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 if (leader) mbar_arrive_expect_tx(&hfull[stage], p.halo_tx);
                 uint8_t *dst = IS4 ? smem + p.off_hp + stage * p.hp_stage_bytes
                                    : smem + p.off_hx + stage * p.hx_stage_bytes;
-                if (leader) tma_load_5d(dst, &hmap, &hfull[stage], 0, -p.pad_w, p0 - p.pad_h, img, 0);
+                if (p.halo_flat) {     // rows of Wh pixels as int64 elements: few long TMA rows
+                    if (leader) tma_load_3d(dst, &hmap, &hfull[stage], -p.pad_w * (p.c_px / 8), p0 - p.pad_h, img);
+                } else {
+                    if (leader) tma_load_5d(dst, &hmap, &hfull[stage], 0, -p.pad_w, p0 - p.pad_h, img, 0);
+                }
             }
         }
     } else if (warp == kWarpMMA) {
@@ -239,14 +243,18 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             const uint32_t dst = smem_u32(smem + p.off_hx + stage * p.hx_stage_bytes);
             constexpr int kStride = kNumCvtWarps * 32;
             constexpr int U = 4;            // loads batched ahead of the conversion
+            // packed 16-byte chunk j of pixel px: plane-major staging (5-D load) or pixel-major
+            // staging (flat load)
+            const uint32_t sstr = p.halo_flat ? static_cast<uint32_t>(p.c_px) : 16u;
             for (int j = 0; j < p.nplanes / 2; ++j) {
-                const uint32_t sj = src + static_cast<uint32_t>(j * npix) * 16u;
+                const uint32_t sj = src + (p.halo_flat ? 16u * static_cast<uint32_t>(j)
+                                                       : static_cast<uint32_t>(j * npix) * 16u);
                 const uint32_t dj = dst + static_cast<uint32_t>(2 * j) * p.h_plane_bytes;
                 int px = ct;
                 for (; px + (U - 1) * kStride < npix; px += U * kStride) {
                     uint4 pk[U];
 #pragma unroll
-                    for (int u = 0; u < U; ++u) pk[u] = lds128u(sj + static_cast<uint32_t>(px + u * kStride) * 16u);
+                    for (int u = 0; u < U; ++u) pk[u] = lds128u(sj + static_cast<uint32_t>(px + u * kStride) * sstr);
 #pragma unroll
                     for (int u = 0; u < U; ++u) {
                         uint32_t o[8];
@@ -260,7 +268,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                     }
                 }
                 for (; px < npix; px += kStride) {
-                    const uint4 pk = lds128u(sj + static_cast<uint32_t>(px) * 16u);
+                    const uint4 pk = lds128u(sj + static_cast<uint32_t>(px) * sstr);
                     uint32_t o[8];
                     widen_word(pk.x, xo, o[0], o[4]);
                     widen_word(pk.y, xo, o[1], o[5]);

@@ -522,6 +522,11 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.off_hp = bres + hx * stages;
     p.hp_stage_bytes = hp;
     p.halo_tx = static_cast<uint32_t>(nch) * plane;
+    // whole-row loads when one box row (Wh pixels) fits the 256-element limit as int64s and the
+    // staged layout works without planes: the C = 16 stem (one plane) or 4-bit inputs (the
+    // converter re-lays the packed pixels into planes)
+    p.c_px = g.c_bytes;
+    p.halo_flat = ((tap_pair || is4) && (Wh * g.c_bytes) % 8 == 0 && Wh * g.c_bytes / 8 <= 256) ? 1 : 0;
     p.off_ystg = static_cast<uint32_t>(align_up(p.off_hp + hp * stages, 1024));
     p.ystg_bytes = ystg / 2;
     p.y_tma = 1;
@@ -559,7 +564,18 @@ qc_status encode_halo_maps(const qconv_desc *d, const Geometry &g, const qc::Con
     const Driver &drv = driver();
     if (!drv.tiled) return cuda_fail(drv.err);
     const cuuint64_t cb = static_cast<cuuint64_t>(g.c_bytes);
-    {   // input halo: [chunk][n][h][w][16 B] view of NHWC
+    if (p.halo_flat) {   // input halo: [n][h][w * c_bytes / 8] int64 view of NHWC, whole rows
+        cuuint64_t dims[3] = {static_cast<cuuint64_t>(d->w) * cb / 8, static_cast<cuuint64_t>(d->h),
+                              static_cast<cuuint64_t>(d->n)};
+        cuuint64_t strides[2] = {cb * d->w, cb * d->w * d->h};
+        cuuint32_t box[3] = {static_cast<cuuint32_t>(p.Wh * cb / 8), static_cast<cuuint32_t>(p.HR), 1};
+        cuuint32_t es[3] = {1, 1, 1};
+        CUresult r = drv.tiled(hm, CU_TENSOR_MAP_DATA_TYPE_INT64, 3, const_cast<void *>(x), dims, strides,
+                               box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+        small_tensor_fixup(hm, static_cast<uint64_t>(g.x_bytes));
+    } else {   // input halo: [chunk][n][h][w][16 B] view of NHWC
         cuuint64_t dims[5] = {16, static_cast<cuuint64_t>(d->w), static_cast<cuuint64_t>(d->h),
                               static_cast<cuuint64_t>(d->n), cb / 16};
         cuuint64_t strides[4] = {cb, cb * d->w, cb * d->w * d->h, 16};
@@ -703,7 +719,7 @@ bool make_trans_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     int grid = static_cast<int>(std::min<int64_t>(num_tiles, sms / n_tiles_n * n_tiles_n));
     grid = std::max(grid, 1);
     pl->grid = grid;
-    pl->threads = is4 ? 512 : 384;
+    pl->threads = is4 ? qc::kTThreads4 : qc::kTThreads8;
     pl->BK = BK; pl->bkp = bkp; pl->BN = BMc; pl->n_tiles_n = n_tiles_n;
     pl->num_tiles = static_cast<int>(num_tiles); pl->stages = stages; pl->chunks = p.chunks;
     pl->num_kb = p.num_kb;

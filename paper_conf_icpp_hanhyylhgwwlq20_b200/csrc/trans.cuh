@@ -51,7 +51,7 @@ __device__ __forceinline__ int32_t t_requant(const ConvParams &p, const TChan &c
 // pixel into the swizzled staging rows.  The swizzle term of row px0 + 8k does not depend on
 // k (rows step by 8, the XOR uses row bits below 8 rows), so the two store addresses are
 // computed once and the repetitions use immediate offsets.
-template <int OUT, int MODE, bool CLAMP, int RB, int GMASK>
+template <int OUT, int MODE, bool CLAMP, int RB, int GMASK, bool ALU_PACK = false>
 __device__ __forceinline__ void t_pairs(const ConvParams &p, const TChan &ce, const TChan &co,
                                         const uint32_t (&v)[32], uint32_t ystg, int row0, uint32_t boff) {
     constexpr bool kInt4 = (OUT == OUT_U4 || OUT == OUT_S4);
@@ -68,7 +68,21 @@ __device__ __forceinline__ void t_pairs(const ConvParams &p, const TChan &ce, co
             yo0 = min(hi, max(lo, yo0)); yo1 = min(hi, max(lo, yo1));
         }
         const uint32_t d = static_cast<uint32_t>(8 * k * RB);
-        if (kInt4) {
+        if (ALU_PACK) {
+            // saturate with min/max and pack with one LEA (ALU pipe) instead of I2IP
+            constexpr int32_t qlo = OUT == OUT_U4 ? 0 : (OUT == OUT_S4 ? -8 : (OUT == OUT_U8 ? 0 : -128));
+            constexpr int32_t qhi = OUT == OUT_U4 ? 15 : (OUT == OUT_S4 ? 7 : (OUT == OUT_U8 ? 255 : 127));
+            constexpr uint32_t msk = kInt4 ? 0xFu : 0xFFu;
+            constexpr int sh = kInt4 ? 4 : 8;
+            if (!CLAMP) {
+                ye0 = min(qhi, max(qlo, ye0)); ye1 = min(qhi, max(qlo, ye1));
+                yo0 = min(qhi, max(qlo, yo0)); yo1 = min(qhi, max(qlo, yo1));
+            }
+            const uint32_t w0 = (static_cast<uint32_t>(yo0) << sh) | (static_cast<uint32_t>(ye0) & msk);
+            const uint32_t w1 = (static_cast<uint32_t>(yo1) << sh) | (static_cast<uint32_t>(ye1) & msk);
+            if (kInt4) { sts8(a0 + d, w0); sts8(a1 + d, w1); }
+            else { sts16(a0 + d, w0); sts16(a1 + d, w1); }
+        } else if (kInt4) {
             sts8(a0 + d, OUT == OUT_U4 ? pack_sat_u4(yo0, ye0, 0u) : pack_sat_s4(yo0, ye0, 0u));
             sts8(a1 + d, OUT == OUT_U4 ? pack_sat_u4(yo1, ye1, 0u) : pack_sat_s4(yo1, ye1, 0u));
         } else {
@@ -117,8 +131,15 @@ __device__ __forceinline__ void t_chan_mid(const ConvParams &p, TChan &c, int ne
     c.c64 = static_cast<int64_t>((1 << (T - 33)) + p.y_zero * (1 << (T - 32))) << 32;
 }
 
+// 16 epilogue warps (4 per SMSP: the re-quantization is latency- not issue-bound), then the
+// 4 converter warps (4-bit).
+constexpr int kTEpiWarps = 16;
+constexpr int kTWarpCvt0 = kWarpEpi0 + kTEpiWarps;
+constexpr int kTThreads8 = 32 * kTWarpCvt0;
+constexpr int kTThreads4 = 32 * (kTWarpCvt0 + kNumCvtWarps);
+
 template <bool IS4, int OUT, bool M64>
-__global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
+__global__ void __launch_bounds__(IS4 ? kTThreads4 : kTThreads8, 1)
 qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap wmap,
                const __grid_constant__ CUtensorMap ymap, const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -152,7 +173,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(&tfull[i], 1);
-            mbar_init(&tempty[i], kNumEpiWarps);
+            mbar_init(&tempty[i], kTEpiWarps);
         }
         fence_mbar_init();
     }
@@ -195,7 +216,8 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         }
     } else if (warp == kWarpMMA) {
         // ===================== MMA issuer: D[c, px] += W[c, :] . X[px, :] =====================
-        if (lane == 0) {
+        // whole warp runs the loop, one elected lane issues (see conv_fwd.cuh)
+        {
             int it = 0, g = 0;
             const uint32_t sbo = 8u * static_cast<uint32_t>(p.BK);
             const int ksteps = p.BK / 32;
@@ -203,42 +225,44 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 const int buf = it & 1;
                 const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
                 mbar_wait(&tempty[buf], acc_phase ^ 1u);
+                __syncwarp();
                 tc_fence_after();
-                trace_ev(p, 2, it);
+                if (lane == 0) trace_ev(p, 2, it);
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * BNp);
                 for (int kb = 0; kb < p.num_kb; ++kb, ++g) {
                     const int stage = g % NS;
                     const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
                     mbar_wait(IS4 ? &aready[stage] : &full[stage], phase);
+                    __syncwarp();
                     tc_fence_after();
-                    trace_ev(p, 3, g);
+                    if (lane == 0) trace_ev(p, 3, g);
                     const uint32_t w_addr = smem_u32(smem + p.off_b + stage * p.b_stage_bytes);
                     const uint32_t x_addr = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
+                    const uint64_t ad0 = make_smem_desc(w_addr, 16u, sbo, p.sw_layout);
+                    const uint64_t bd0 = make_smem_desc(x_addr, 16u, sbo, p.sw_layout);
                     for (int k = 0; k < ksteps; ++k) {
-                        const uint64_t ad = make_smem_desc(w_addr + 32u * k, 16u, sbo, p.sw_layout);
-                        const uint64_t bd = make_smem_desc(x_addr + 32u * k, 16u, sbo, p.sw_layout);
                         if (!(p.exp_flags & 4) || (kb | k) == 0)
-                            mma_i8(d_tmem, ad, bd, p.idesc, (kb | k) != 0 ? 1u : 0u);
+                            mma_i8_warp(d_tmem, ad0 + 2u * k, bd0 + 2u * k, p.idesc, (kb | k) != 0 ? 1u : 0u);
                     }
-                    mma_commit(&empty[stage]);
+                    mma_commit_warp(&empty[stage]);
                 }
-                mma_commit(&tfull[buf]);
-                trace_ev(p, 4, it);
+                mma_commit_warp(&tfull[buf]);
+                if (lane == 0) trace_ev(p, 4, it);
             }
         }
-    } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kNumEpiWarps) {
+    } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kTEpiWarps) {
         // ===================== epilogue: lane = output channel, thread = channel pair ===========
         const int ew = warp - kWarpEpi0;
         const int quarter = warp & 3;
-        const int half = ew >> 2;
-        // 16-lane group of this warp and its pixel range.  M=128: quarter q holds groups 2q, 2q+1
-        // (one per warp), all 256 pixels.  M=64 (1-CTA): rows live in lanes 0..15 of each quarter
-        // (group q), the two warps of a quarter split the pixels.
-        const int grp = M64 ? quarter : 2 * quarter + half;
+        const int sub = ew >> 2;                           // 0..3: the 4 warps of a lane quarter
+        // 16-lane group of this warp and its pixel range.  M=128: quarter q holds groups 2q, 2q+1,
+        // two warps per group, 128 pixels each.  M=64 (1-CTA): rows live in lanes 0..15 of each
+        // quarter (group q), the four warps of a quarter take 64 pixels each.
+        const int grp = M64 ? quarter : 2 * quarter + (sub & 1);
         const uint32_t lane_base = M64 ? 32u * static_cast<uint32_t>(quarter)
-                                       : 32u * static_cast<uint32_t>(quarter) + 16u * static_cast<uint32_t>(half);
-        constexpr int kCols = M64 ? kBNp / 2 : kBNp;
-        const int col_begin = M64 ? half * kCols : 0;
+                                       : 32u * static_cast<uint32_t>(quarter) + 16u * static_cast<uint32_t>(sub & 1);
+        constexpr int kCols = M64 ? kBNp / 4 : kBNp / 2;
+        const int col_begin = M64 ? sub * kCols : (sub >> 1) * kCols;
         const int pair = 8 * grp + (lane >> 2);             // channel pair of the tile
         constexpr int kGMask = kRowBytes >= 128 ? 7 : (kRowBytes == 64 ? 3 : 1);
         const uint32_t boff = static_cast<uint32_t>(kInt4 ? pair : 2 * pair);
@@ -275,38 +299,32 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             const uint32_t taddr = tmem_base + (lane_base << 16) + static_cast<uint32_t>(buf * kBNp + col_begin);
             const bool storer = ew == 0 && lane == 0;
             if (storer) bulk_wait_read<1>();
-            named_bar_sync(1, kNumEpiWarps * 32);
+            named_bar_sync(1, kTEpiWarps * 32);
             const uint32_t ystg = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes;
             const int row0 = col_begin + 2 * (lane & 3);
-            // 64-pixel chunks, TMEM loads double-buffered against the requantization
-            uint32_t va[32], vb[32];
-            tmem_ld_16x256b_x8(taddr, va);
-#pragma unroll
-            for (int t = 0; t < kCols / 64; t += 2) {
+            // 64-pixel chunks (latency hidden by the 4 epilogue warps per SMSP)
+#pragma unroll 1
+            for (int t = 0; t < kCols / 64; ++t) {
+                uint32_t va[32];
+                tmem_ld_16x256b_x8(taddr + static_cast<uint32_t>(t * 64), va);
                 tmem_wait_ld_regs(va);
-                if (t + 1 < kCols / 64) tmem_ld_16x256b_x8(taddr + static_cast<uint32_t>((t + 1) * 64), vb);
                 t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, va, ystg, row0 + 64 * t, boff);
-                if (t + 1 < kCols / 64) {
-                    tmem_wait_ld_regs(vb);
-                    if (t + 2 < kCols / 64) tmem_ld_16x256b_x8(taddr + static_cast<uint32_t>((t + 2) * 64), va);
-                    t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, vb, ystg, row0 + 64 * (t + 1), boff);
-                }
             }
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(&tempty[buf]);
             if (ew == 0 && lane == 0) trace_ev(p, 6, it);
             fence_proxy_async_smem();
-            named_bar_sync(1, kNumEpiWarps * 32);
+            named_bar_sync(1, kTEpiWarps * 32);
             if (storer && !(p.exp_flags & 128)) {
                 tma_store_2d(&ymap, smem + p.off_ystg + (it & 1) * p.ystg_bytes, c0 * (kInt4 ? 4 : 8) / 8, m0);
                 bulk_commit();
             }
         }
         if (ew == 0 && lane == 0) bulk_wait<0>();
-    } else if (IS4 && warp >= kWarpCvt0 && warp < kWarpCvt0 + kNumCvtWarps) {
+    } else if (IS4 && warp >= kTWarpCvt0 && warp < kTWarpCvt0 + kNumCvtWarps) {
         // ===================== int4 -> int8 widening of the activation tile =====================
-        const int ct = (warp - kWarpCvt0) * 32 + lane;
+        const int ct = (warp - kTWarpCvt0) * 32 + lane;
         const int cshift = p.cvt_shift;
         const int nchunks = BNp << cshift;
         const uint32_t xo = p.x_sgn4 ? 0x88888888u : 0u;
