@@ -64,6 +64,11 @@ struct ConvParams {
     int32_t halo_flat;                // halo loaded as whole pixel rows (3-D int64 view): staged
                                       // pixel-major [HR][Wh][c_px bytes] instead of 16-byte planes
     int32_t c_px;                     // packed bytes per input pixel (halo_flat)
+    int32_t w_early;                  // weights may be loaded before griddep_wait (they were not
+                                      // written by a kernel of this call)
+    int32_t stg_sw;                   // TMA swizzle mask of the packed 4-bit staging rows (0 none,
+                                      // 1 32B, 3 64B, 7 128B): SWIZZLE_NONE loads move 16 B per
+                                      // request and are several times slower than swizzled ones
     uint32_t off_mtab; int32_t n_mma;  // halo: per-MMA descriptor offsets {a>>4, b>>4}
     // shared memory carve-up (byte offsets from the 1024-aligned base)
     uint32_t off_a, off_b, off_stg, off_bar, off_par;
@@ -403,7 +408,8 @@ __device__ __forceinline__ void widen_word(uint32_t w, uint32_t xo, uint32_t &lo
 // the destination offsets are computed once.  Four chunks are loaded before any is
 // converted so the shared-memory latency overlaps.
 __device__ __forceinline__ void widen_stage(uint32_t stg, uint32_t adst, int ct, int nchunks,
-                                            int cshift, uint32_t bkb, uint32_t sw, uint32_t xo) {
+                                            int cshift, uint32_t bkb, uint32_t sw, uint32_t xo,
+                                            uint32_t ssw) {
     constexpr int kStride = kNumCvtWarps * 32;
     constexpr int U = 4;
     const uint32_t rr = static_cast<uint32_t>(ct) >> cshift;
@@ -413,7 +419,10 @@ __device__ __forceinline__ void widen_stage(uint32_t stg, uint32_t adst, int ct,
     const uint32_t d0 = adst + (off0 ^ (((off0 >> 7) & sw) << 4));
     const uint32_t d1 = adst + (off1 ^ (((off1 >> 7) & sw) << 4));
     const uint32_t dstep = (static_cast<uint32_t>(kStride) >> cshift) * bkb;
-    const uint32_t s0 = stg + 16u * static_cast<uint32_t>(ct);
+    // source chunk in the (TMA-swizzled) packed staging; the XOR term is the same for all of
+    // this thread's chunks (they are >= 32 rows apart)
+    const uint32_t soff = 16u * static_cast<uint32_t>(ct);
+    const uint32_t s0 = stg + (soff ^ (((soff >> 7) & ssw) << 4));
     int i = 0;
     const int n_mine = ct < nchunks ? (nchunks - ct + kStride - 1) / kStride : 0;
     for (; i + U <= n_mine; i += U) {
@@ -466,6 +475,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
     EpiCol *par = reinterpret_cast<EpiCol *>(smem + p.off_par);
     int4 *chunk_info = reinterpret_cast<int4 *>(smem + p.off_par + 16 * kMaxBN);  // [8] {mode, rhiT, shT, 0}
 
+    griddep_launch_dependents();
     if (warp == kWarpTMA && lane == 0) {
         tma_prefetch_desc(&xmap);
         tma_prefetch_desc(&wmap);
@@ -495,6 +505,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
         // 16 KB), so K-stages are dealt round-robin to kNumProducers threads.
         if (lane == 0) {   // one thread issues (measured faster than an elected warp-wide loop)
             constexpr bool leader = true;
+            griddep_wait();                                         // activations of the previous layer
             const int pi = warp == kWarpTMA ? 0 : warp - 1;       // 0, 1, 2
             const uint32_t tx = static_cast<uint32_t>(kBM * (p.pair ? 32 : p.bkp) + p.BN * p.BK);
             int g = 0;                                              // CTA-local K-stage counter
@@ -601,6 +612,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
         }
     } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kNumEpiWarps) {
         // ===================== epilogue (8 warps: lane quarter = warp%4, column half) ============
+        griddep_wait();                                   // params / tables written in-stream
         const int ew = warp - kWarpEpi0;                 // 0..7
         const int quarter = warp & 3;                    // TMEM lanes 32*quarter .. +31
         const int half = ew >> 2;                        // which 32-column chunks
@@ -740,7 +752,7 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 if (ct == 0) trace_ev(p, 8, cstage++);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
-                widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo);
+                widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
                 fence_proxy_async_smem();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&aready[stage]);

@@ -43,6 +43,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
     EpiCol *par = reinterpret_cast<EpiCol *>(smem + p.off_par);
     int4 *chunk_info = reinterpret_cast<int4 *>(smem + p.off_par + 16 * kMaxBN);
 
+    griddep_launch_dependents();
     if (warp == kWarpTMA && lane == 0) {
         tma_prefetch_desc(&hmap);
         tma_prefetch_desc(&bmap);
@@ -71,8 +72,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         // ===================== TMA producer =====================
         if (lane == 0) {   // one thread issues (measured faster than an elected warp-wide loop)
             constexpr bool leader = true;
+            if (!p.w_early) griddep_wait();                         // weights prepared in this call
             if (leader) mbar_arrive_expect_tx(bfull, p.b_res_bytes);
             if (leader) tma_load_3d(smem + p.off_bres, &bmap, bfull, 0, n0, 0);
+            if (p.w_early) griddep_wait();                          // activations of the previous layer
             int g = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
                 const int mt = tile / p.n_tiles_n;
@@ -119,6 +122,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 if (leader) trace_ev(p, 3, it);
                 __syncwarp();
                 tc_fence_after();
+                if (leader) trace_ev(p, 1, it);
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
                 const uint64_t adesc0 = make_smem_desc(smem_u32(smem + p.off_hx + stage * p.hx_stage_bytes),
                                                        a_lbo, 128u, 0u);
@@ -129,7 +133,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                         uint64_t ad = adesc0 + static_cast<uint32_t>(r * p.Wh + s);
                         uint64_t bd = bdesc0 + (p.tap_pair ? tap : tap * static_cast<uint32_t>(p.nplanes)) * b_pl16;
                         for (int j = 0; j < npl; j += 2) {
-                            if (!(p.exp_flags & 4) || acc == 0u)    // debug ablation: one MMA per tile
+                            if ((!(p.exp_flags & 4) || acc == 0u) && !(p.exp_flags & 64))   // debug ablations
                                 mma_i8_warp(d_tmem, ad, bd, p.idesc, acc);
                             acc = 1u;
                             ad += 2u * a_pl16;
@@ -137,13 +141,16 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                         }
                     }
                 }
+                if (leader) trace_ev(p, 11, it);
                 mma_commit_warp(&hempty[stage]);
+                if (leader) trace_ev(p, 12, it);
                 mma_commit_warp(&tfull[buf]);
                 if (leader) trace_ev(p, 4, it);
             }
         }
     } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kNumEpiWarps) {
         // ===================== epilogue =====================
+        griddep_wait();                                   // params written in-stream
         const int ew = warp - kWarpEpi0;
         const int quarter = warp & 3;
         const int half = ew >> 2;
@@ -217,7 +224,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             if (ew == 0 && lane == 0) trace_ev(p, 6, it);
             fence_proxy_async_smem();
             named_bar_sync(1, kNumEpiWarps * 32);
-            if (storer) {
+            if (storer && !(p.exp_flags & 128)) {
                 constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
                 for (int gi = 0; gi < p.n_ygroups; ++gi)
                     tma_store_4d(&ymap, smem + p.off_ystg + (it & 1) * p.ystg_bytes + gi * 128 * p.y_gw,

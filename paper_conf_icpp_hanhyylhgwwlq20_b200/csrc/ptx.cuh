@@ -86,6 +86,17 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     }
 }
 
+// ---------------------------------------------------------------- programmatic dependent launch
+// The conv kernels are launched with programmatic stream serialization: a kernel may start
+// (prologue, barrier init, TMEM alloc, descriptor prefetch, weight loads) while the previous
+// kernel of the stream drains.  Every thread that reads activations produced by an earlier
+// kernel (the TMA producers) first waits for the prerequisite grid to complete; everything
+// else that touches global memory is ordered after those loads by the pipeline.
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void griddep_launch_dependents() {
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // ---------------------------------------------------------------- fences / barriers
 __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");

@@ -309,6 +309,16 @@ CUtensorMapSwizzle swizzle_for(int bk) {
                      : (bk == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B);
 }
 
+// Packed 4-bit staging rows of `bytes` per pixel are loaded swizzled whenever the row width
+// allows (32/64/128 B): SWIZZLE_NONE boxes are moved in 16-byte requests, several times slower
+// (measured: conv1/halo ablations, r1).  The converter reads the swizzled layout (widen_stage).
+CUtensorMapSwizzle packed_swizzle(int bytes) {
+    return bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                        : (bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                       : (bytes == 32 ? CU_TENSOR_MAP_SWIZZLE_32B : CU_TENSOR_MAP_SWIZZLE_NONE));
+}
+int packed_sw_mask(int bytes) { return bytes == 128 ? 7 : (bytes == 64 ? 3 : (bytes == 32 ? 1 : 0)); }
+
 qc_status encode_x_map(const qconv_desc *d, const Geometry &g, const void *x, int box_bytes,
                        CUtensorMapSwizzle sw, CUtensorMap *map, int pixels = qc::kBM) {
     const Driver &drv = driver();
@@ -385,6 +395,17 @@ qc_status encode_y_map(const qconv_desc *d, const Geometry &g, void *y, int gw, 
     return QC_OK;
 }
 
+// Programmatic dependent launch (see ptx.cuh griddep_wait): the conv kernels may start while
+// the previous kernel of the stream drains; QC_NO_PDL=1 disables it (debug).
+void set_pdl(cudaLaunchConfig_t &cfg, cudaLaunchAttribute *attr) {
+    static const bool off = std::getenv("QC_NO_PDL") != nullptr;
+    if (off) return;
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+}
+
 // Debug hooks (never set in normal use): QC_EXPERIMENT=<flags> ablations, and
 // QC_TRACE=<file> timestamps of CTA 0's pipeline events, appended to the file after a sync.
 qc::ConvParams debug_params(const qc::ConvParams &base, cudaStream_t stream) {
@@ -431,8 +452,8 @@ qc_status launch_conv_t(const Plan &pl, const CUtensorMap &xm, const CUtensorMap
     cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
     cfg.dynamicSmemBytes = pl.smem_bytes;
     cfg.stream = stream;
-    cfg.attrs = nullptr;
-    cfg.numAttrs = 0;
+    cudaLaunchAttribute pdl[1];
+    set_pdl(cfg, pdl);
     qc::ConvParams cp = debug_params(pl.cp, stream);
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
     if (e != cudaSuccess) return cuda_fail(e);
@@ -504,7 +525,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
                            8u * static_cast<uint32_t>(d->r * d->s * nplanes);
     if (fixed + 2 * (hx + hp) > 227u * 1024u) return false;
     int stages = static_cast<int>((227u * 1024u - fixed) / (hx + hp));
-    stages = std::min(stages, 6);
+    stages = std::min(stages, 24);   // deep ring: the halo loads are latency-bound (~6 us each under load)
     qc::ConvParams &p = pl->cp;
     std::memset(&p, 0, sizeof(p));
     p.M = static_cast<int32_t>(g.M);
@@ -634,6 +655,8 @@ qc_status launch_halo(const Plan &pl, const CUtensorMap &hm, const CUtensorMap &
     cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
     cfg.dynamicSmemBytes = pl.smem_bytes;
     cfg.stream = stream;
+    cudaLaunchAttribute pdl[1];
+    set_pdl(cfg, pdl);
     qc::ConvParams cp = debug_params(pl.cp, stream);
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, hm, bm, ym, cp);
     if (e != cudaSuccess) return cuda_fail(e);
@@ -742,6 +765,8 @@ qc_status launch_trans_m(const Plan &pl, const CUtensorMap &xm, const CUtensorMa
     cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
     cfg.dynamicSmemBytes = pl.smem_bytes;
     cfg.stream = stream;
+    cudaLaunchAttribute pdl[1];
+    set_pdl(cfg, pdl);
     qc::ConvParams cp = debug_params(pl.cp, stream);
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
     if (e != cudaSuccess) return cuda_fail(e);
@@ -947,6 +972,7 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
         Plan hp;
         if (need_z == 0 && make_halo_plan(d, g, &hp)) {
             set_act_params(d, g, w8, hp.cp);
+            hp.cp.w_early = need_w == 0 ? 1 : 0;
             hp.cp.bias = bias;
             hp.cp.mult = multiplier;
             hp.cp.shift = shift;
@@ -973,7 +999,8 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
             tp.cp.shift = shift;
             tp.cp.y = y;
             alignas(64) CUtensorMap xm, wm, ym;
-            s = encode_x_map(d, g, x, tp.bkp, g.bits == 4 ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(tp.BK), &xm,
+            tp.cp.stg_sw = g.bits == 4 ? packed_sw_mask(tp.bkp) : 0;
+            s = encode_x_map(d, g, x, tp.bkp, g.bits == 4 ? packed_swizzle(tp.bkp) : swizzle_for(tp.BK), &xm,
                              tp.cp.Wh);
             if (s != QC_OK) return s;
             s = encode_w_map_pairs(d, g, w8, tp.BK, tp.BN, swizzle_for(tp.BK), &wm);
@@ -1008,8 +1035,10 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
 
     alignas(64) CUtensorMap xm, wm;
     const bool pair = p.pair != 0;
+    p.stg_sw = g.bits == 4 ? packed_sw_mask(pl.bkp) : 0;
     s = encode_x_map(d, g, x, pl.bkp,
-                     (g.bits == 4 || pair) ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(pl.BK), &xm);
+                     pair ? CU_TENSOR_MAP_SWIZZLE_NONE : (g.bits == 4 ? packed_swizzle(pl.bkp) : swizzle_for(pl.BK)),
+                     &xm);
     if (s != QC_OK) return s;
     s = encode_w_map(d, g, w8, pair ? 16 : pl.BK, pl.BN,
                      pair ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(pl.BK), &wm);

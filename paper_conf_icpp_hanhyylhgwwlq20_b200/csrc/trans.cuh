@@ -162,6 +162,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
     uint64_t *tempty = bars + 3 * NS + 2;
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 4);
 
+    griddep_launch_dependents();
     if (warp == kWarpTMA && lane == 0) {
         tma_prefetch_desc(&xmap);
         tma_prefetch_desc(&wmap);
@@ -186,6 +187,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
     if (warp == kWarpTMA || warp == 2 || warp == 3) {
         // ===================== TMA producers =====================
         if (lane == 0) {
+            griddep_wait();                                         // activations of the previous layer
             const int pi = warp == kWarpTMA ? 0 : warp - 1;
             const uint32_t tx = static_cast<uint32_t>(BNp * p.bkp + BMc * p.BK);
             int g = 0;
@@ -252,6 +254,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         }
     } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kTEpiWarps) {
         // ===================== epilogue: lane = output channel, thread = channel pair ===========
+        griddep_wait();                                   // params written in-stream
         const int ew = warp - kWarpEpi0;
         const int quarter = warp & 3;
         const int sub = ew >> 2;                           // 0..3: the 4 warps of a lane quarter
@@ -339,7 +342,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 if (ct == 0) trace_ev(p, 8, g);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
-                if (!(p.exp_flags & 8)) widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo);
+                if (!(p.exp_flags & 8)) widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
                 if (ct == 0) trace_ev(p, 10, g);
                 fence_proxy_async_smem();
                 __syncwarp();

@@ -12,8 +12,8 @@ import torch
 import bench
 tr = bench.Trunk(bits, 256, "cuda")
 import paper_conf_icpp_hanhyylhgwwlq20_b200 as qc
-EV = ["prod_issue", "-", "mma_tempty_ok", "mma_full_ok", "mma_commit", "epi_tfull_ok", "epi_tempty_arrive",
-      "epi_store_issued", "cvt_full_ok", "cvt_done", "cvt_loop_done"]
+EV = ["prod_issue", "mma_fenced", "mma_tempty_ok", "mma_full_ok", "mma_commit", "epi_tfull_ok", "epi_tempty_arrive",
+      "epi_store_issued", "cvt_full_ok", "cvt_done", "cvt_loop_done", "mma_issued", "mma_commit1"]
 for L in tr.layers:
     if L["name"] not in names:
         continue
