@@ -21,6 +21,8 @@
 
 namespace qc {
 
+constexpr int kHaloMaxMMA = 18;      // 3x3 taps x 2 plane pairs (C = 64), or the 4x4/2 stem pairs
+
 template <bool IS4, int OUT>
 __global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
 qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap bmap,
@@ -107,6 +109,23 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             const int npl = p.tap_pair ? 1 : p.nplanes;
             const uint64_t bdesc0 = make_smem_desc(smem_u32(smem + p.off_bres), bplane, 128u, 0u);
             const uint32_t a_lbo = p.tap_pair ? 16u : p.h_plane_bytes;
+            // per-MMA descriptor offsets (16-byte units), K order = (r, s, plane pair)
+            uint32_t aoff[kHaloMaxMMA], boff[kHaloMaxMMA];
+            const int nmma = p.n_mma;
+            {
+                int r = 0, sx = 0, j = 0;
+#pragma unroll
+                for (int i = 0; i < kHaloMaxMMA; ++i) {
+                    const uint32_t tap = static_cast<uint32_t>(r * p.S + sx);
+                    aoff[i] = static_cast<uint32_t>(r * p.Wh + sx) + static_cast<uint32_t>(j) * a_pl16;
+                    boff[i] = (p.tap_pair ? tap : tap * static_cast<uint32_t>(p.nplanes) + static_cast<uint32_t>(j)) * b_pl16;
+                    j += 2;
+                    if (j >= npl) { j = 0; sx += sstep; if (sx >= p.S) { sx = 0; ++r; } }
+                }
+            }
+            const uint64_t adesc_st = make_smem_desc(smem_u32(smem + p.off_hx), a_lbo, 128u, 0u);
+            const uint32_t ahi = static_cast<uint32_t>(adesc_st >> 32);
+            const uint32_t blo0 = static_cast<uint32_t>(bdesc0), bhi = static_cast<uint32_t>(bdesc0 >> 32);
             mbar_wait(bfull, 0);
             __syncwarp();
             tc_fence_after();
@@ -124,22 +143,13 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 tc_fence_after();
                 if (leader) trace_ev(p, 1, it);
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
-                const uint64_t adesc0 = make_smem_desc(smem_u32(smem + p.off_hx + stage * p.hx_stage_bytes),
-                                                       a_lbo, 128u, 0u);
-                uint32_t acc = 0u;
-                for (int r = 0; r < p.R; ++r) {
-                    for (int s = 0; s < p.S; s += sstep) {
-                        const uint32_t tap = static_cast<uint32_t>(r * p.S + s);
-                        uint64_t ad = adesc0 + static_cast<uint32_t>(r * p.Wh + s);
-                        uint64_t bd = bdesc0 + (p.tap_pair ? tap : tap * static_cast<uint32_t>(p.nplanes)) * b_pl16;
-                        for (int j = 0; j < npl; j += 2) {
-                            if ((!(p.exp_flags & 4) || acc == 0u) && !(p.exp_flags & 64))   // debug ablations
-                                mma_i8_warp(d_tmem, ad, bd, p.idesc, acc);
-                            acc = 1u;
-                            ad += 2u * a_pl16;
-                            bd += 2u * b_pl16;
-                        }
-                    }
+                const uint32_t alo0 = static_cast<uint32_t>(adesc_st) +
+                                      ((static_cast<uint32_t>(stage) * p.hx_stage_bytes) >> 4);
+                // fully unrolled over the precomputed per-MMA offsets (registers)
+#pragma unroll
+                for (int i = 0; i < kHaloMaxMMA; ++i) {
+                    if (i < nmma && (!(p.exp_flags & 4) || i == 0) && !(p.exp_flags & 64))   // debug ablations
+                        mma_i8_warp_lo(d_tmem, alo0 + aoff[i], ahi, blo0 + boff[i], bhi, p.idesc, i > 0 ? 1u : 0u);
                 }
                 if (leader) trace_ev(p, 11, it);
                 mma_commit_warp(&hempty[stage]);

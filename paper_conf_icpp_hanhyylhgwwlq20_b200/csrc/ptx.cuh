@@ -242,6 +242,20 @@ __device__ __forceinline__ void mma_i8_warp(uint32_t d_tmem, uint64_t adesc, uin
         "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
         : "memory");
 }
+// Same, with the descriptors' high words fixed and only the low words (start address,
+// LBO) passed per MMA: no 64-bit adds in the issue loop.
+__device__ __forceinline__ void mma_i8_warp_lo(uint32_t d_tmem, uint32_t alo, uint32_t ahi, uint32_t blo,
+                                               uint32_t bhi, uint32_t idesc, uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p, e;\n\t.reg .b64 da, db;\n\t"
+        "setp.ne.b32 p, %7, 0;\n\t"
+        "mov.b64 da, {%1, %2};\n\t"
+        "mov.b64 db, {%3, %4};\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::i8 [%0], da, db, %5, p;\n\t}" ::"r"(d_tmem),
+        "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "r"(0), "r"(accumulate)
+        : "memory");
+}
 __device__ __forceinline__ void mma_commit_warp(uint64_t *bar) {
     asm volatile(
         "{\n\t.reg .pred e;\n\t"

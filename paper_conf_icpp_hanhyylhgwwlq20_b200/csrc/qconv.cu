@@ -556,6 +556,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.n_ygroups = tile_row_bytes / y_gw;
     p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + ystg, 16));
     p.n_mma = tap_pair ? d->r * (d->s / 2) : d->r * d->s * (nplanes / 2);
+    if (p.n_mma > qc::kHaloMaxMMA) return false;
     p.off_mtab = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u, 16));
     p.off_bar = static_cast<uint32_t>(align_up(p.off_mtab + 8u * static_cast<uint32_t>(p.n_mma), 8));
     const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 5) * 8 + 16);
