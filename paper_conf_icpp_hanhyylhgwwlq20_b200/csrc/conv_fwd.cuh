@@ -598,9 +598,19 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                     } else {
                         const uint64_t ad0 = make_smem_desc(a_addr, 16u, sbo, p.sw_layout);
                         const uint64_t bd0 = make_smem_desc(b_addr, 16u, sbo, p.sw_layout);
-                        for (int k = 0; k < ksteps; ++k) {
-                            if (!(p.exp_flags & 4) || (kb | k) == 0)
-                                mma_i8_warp(d_tmem, ad0 + 2u * k, bd0 + 2u * k, p.idesc, (kb | k) != 0 ? 1u : 0u);
+                        const uint32_t alo = static_cast<uint32_t>(ad0), ahi = static_cast<uint32_t>(ad0 >> 32);
+                        const uint32_t blo = static_cast<uint32_t>(bd0), bhi = static_cast<uint32_t>(bd0 >> 32);
+                        if (ksteps == 4) {
+#pragma unroll
+                            for (int k = 0; k < 4; ++k)
+                                if (!(p.exp_flags & 4) || (kb | k) == 0)
+                                    mma_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
+                                                   (kb | k) != 0 ? 1u : 0u);
+                        } else {
+                            for (int k = 0; k < ksteps; ++k)
+                                if (!(p.exp_flags & 4) || (kb | k) == 0)
+                                    mma_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
+                                                   (kb | k) != 0 ? 1u : 0u);
                         }
                     }
                     mma_commit_warp(&empty[stage]);
