@@ -49,6 +49,19 @@ def load_peaks():
                 source="fallback (B200_PROFILING.md; int8 = 2 x bf16)")
 
 
+def measured_traffic(bits: int, batch: int):
+    """DRAM bytes (read + write) of the 53 conv launches of one step, from the newest ncu
+    launch list summarised under profiles/ (only for the configuration it was measured on)."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_traffic.json")))
+    for fn in reversed(files):
+        with open(fn) as f:
+            d = json.load(f)
+        if d.get("bits", 4) == bits and d.get("batch", 256) == batch:
+            return d["conv_dram_bytes_per_step"]
+    return None
+
+
 # ----------------------------------------------------------------------------- trunk
 def trunk_layers(bits: int, batch: int):
     """(ConvShape, stored C, layer index) in network order for the bench trunk."""
@@ -544,7 +557,9 @@ def main():
             "roofline": {"bound": "tensor", "kernel": "the 53 conv launches (qconv_halo/qconv_t/qconv_fwd kernels)",
                          "achieved": achieved_tops, "peak": peaks["int8_tops_sustained"],
                          "unit": "TOPS", "frac": achieved_tops / peaks["int8_tops_sustained"],
-                         "traffic": None, "peak_source": peaks["source"] + ", sustained",
+                         "traffic": measured_traffic(args.bits, per_gpu),
+                         "traffic_unit": "DRAM bytes per step over the 53 conv launches (ncu, profiles/)",
+                         "peak_source": peaks["source"] + ", sustained",
                          "conv_share_of_step": conv_total_ms / instr_ms_per_step,
                          "launch_times": "CUDA events after every launch, second pass of K instrumented "
                                          "graph replays right after the timed region",
