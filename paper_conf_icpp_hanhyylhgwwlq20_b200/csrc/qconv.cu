@@ -729,7 +729,7 @@ bool make_trans_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.n_ygroups = 1;
     p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + 2u * ystg_one, 16));
     p.off_bar = static_cast<uint32_t>(align_up(p.off_par, 8));
-    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 4) * 8 + 16);
+    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 8) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
     if (pl->smem_bytes > 227u * 1024u) return false;
     p.idesc = qc::make_idesc_i8(static_cast<uint32_t>(BMc), static_cast<uint32_t>(BNp),

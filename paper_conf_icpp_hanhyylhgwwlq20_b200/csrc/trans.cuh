@@ -160,7 +160,9 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
     uint64_t *aready = bars + 2 * NS;
     uint64_t *tfull = bars + 3 * NS;
     uint64_t *tempty = bars + 3 * NS + 2;
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 4);
+    uint64_t *sfull = bars + 3 * NS + 4;    // [2] epilogue warps -> storer: staging buffer written
+    uint64_t *sfree = bars + 3 * NS + 6;    // [2] storer -> epilogue warps: its TMA store has read it
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 8);
 
     griddep_launch_dependents();
     if (warp == kWarpTMA && lane == 0) {
@@ -175,6 +177,8 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         for (int i = 0; i < 2; ++i) {
             mbar_init(&tfull[i], 1);
             mbar_init(&tempty[i], kTEpiWarps);
+            mbar_init(&sfull[i], kTEpiWarps);
+            mbar_init(&sfree[i], 1);
         }
         fence_mbar_init();
     }
@@ -185,6 +189,26 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
     const uint32_t tmem_base = *tmem_slot;
 
     if (warp == kWarpTMA || warp == 2 || warp == 3) {
+        // ===================== output storer (warp 2, lane 1) =====================
+        // The epilogue warps never wait for each other: each arrives on sfull[b] once its part
+        // of staging buffer b is written; this thread waits for all 16, issues the TMA store, and
+        // releases the other buffer (sfree) once the store issued before has read it.
+        if (warp == 2 && lane == 1) {
+            int it = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+                const int b = it & 1;
+                const int m0 = (tile / p.n_tiles_n) * BNp;
+                const int c0 = (tile % p.n_tiles_n) * BMc;
+                mbar_wait(&sfull[b], static_cast<uint32_t>(it >> 1) & 1u);
+                if (!(p.exp_flags & 128))
+                    tma_store_2d(&ymap, smem + p.off_ystg + b * p.ystg_bytes, c0 * (kInt4 ? 4 : 8) / 8, m0);
+                bulk_commit();
+                bulk_wait_read<1>();                 // the store from buffer b^1 has read its smem
+                if (it > 0) mbar_arrive(&sfree[b ^ 1]);
+                trace_ev(p, 7, it);
+            }
+            bulk_wait<0>();
+        }
         // ===================== TMA producers =====================
         if (lane == 0) {
             griddep_wait();                                         // activations of the previous layer
@@ -310,9 +334,8 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             tc_fence_after();
             if (ew == 0 && lane == 0) trace_ev(p, 5, it);
             const uint32_t taddr = tmem_base + (lane_base << 16) + static_cast<uint32_t>(buf * kBNp + col_begin);
-            const bool storer = ew == 0 && lane == 0;
-            if (storer) bulk_wait_read<1>();
-            named_bar_sync(1, kTEpiWarps * 32);
+            // staging buffer it&1 is free once the store of tile it-2 has read it
+            mbar_wait(&sfree[it & 1], (static_cast<uint32_t>(it >> 1) & 1u) ^ 1u);
             const uint32_t ystg = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes;
             const int row0 = col_begin + 2 * (lane & 3);
             // 64-pixel chunks (latency hidden by the 4 epilogue warps per SMSP)
@@ -324,17 +347,14 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, va, ystg, row0 + 64 * t, boff);
             }
             tc_fence_before();
+            fence_proxy_async_smem();                 // staging writes -> visible to the TMA store
             __syncwarp();
-            if (lane == 0) mbar_arrive(&tempty[buf]);
-            if (ew == 0 && lane == 0) trace_ev(p, 6, it);
-            fence_proxy_async_smem();
-            named_bar_sync(1, kTEpiWarps * 32);
-            if (storer && !(p.exp_flags & 128)) {
-                tma_store_2d(&ymap, smem + p.off_ystg + (it & 1) * p.ystg_bytes, c0 * (kInt4 ? 4 : 8) / 8, m0);
-                bulk_commit();
+            if (lane == 0) {
+                mbar_arrive(&tempty[buf]);
+                mbar_arrive(&sfull[it & 1]);
             }
+            if (ew == 0 && lane == 0) trace_ev(p, 6, it);
         }
-        if (ew == 0 && lane == 0) bulk_wait<0>();
     } else if (IS4 && warp >= kTWarpCvt0 && warp < kTWarpCvt0 + kNumCvtWarps) {
         // ===================== int4 -> int8 widening of the activation tile =====================
         const int ct = (warp - kTWarpCvt0) * 32 + lane;
