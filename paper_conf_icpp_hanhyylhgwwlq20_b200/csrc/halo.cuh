@@ -41,7 +41,9 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
     uint64_t *tfull = bars + 3 * NS;        // [2]
     uint64_t *tempty = bars + 3 * NS + 2;   // [2]
     uint64_t *bfull = bars + 3 * NS + 4;    // [1] resident weights landed
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 5);
+    uint64_t *sfull = bars + 3 * NS + 5;    // [2] epilogue warps -> storer: staging buffer written
+    uint64_t *sfree = bars + 3 * NS + 7;    // [2] storer -> epilogue warps: its TMA store has read it
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 9);
     EpiCol *par = reinterpret_cast<EpiCol *>(smem + p.off_par);
     int4 *chunk_info = reinterpret_cast<int4 *>(smem + p.off_par + 16 * kMaxBN);
 
@@ -58,6 +60,8 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         for (int i = 0; i < 2; ++i) {
             mbar_init(&tfull[i], 1);
             mbar_init(&tempty[i], kNumEpiWarps);
+            mbar_init(&sfull[i], kNumEpiWarps);
+            mbar_init(&sfree[i], 1);
         }
         mbar_init(bfull, 1);
         fence_mbar_init();
@@ -70,7 +74,30 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
     // all tiles of this CTA share one N tile (grid is a multiple of n_tiles_n)
     const int n0 = (static_cast<int>(blockIdx.x) % p.n_tiles_n) * p.BN;
 
-    if (warp == kWarpTMA) {
+    if (warp == 2) {
+        // ===================== output storer (see trans.cuh) =====================
+        if (lane == 0) {
+            int it = 0;
+            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+                const int b = it & 1;
+                const int mt = tile / p.n_tiles_n;
+                const int img = mt / p.tiles_per_img;
+                const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
+                mbar_wait(&sfull[b], static_cast<uint32_t>(it >> 1) & 1u);
+                if (!(p.exp_flags & 128)) {
+                    constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
+                    for (int gi = 0; gi < p.n_ygroups; ++gi)
+                        tma_store_4d(&ymap, smem + p.off_ystg + b * p.ystg_bytes + gi * 128 * p.y_gw,
+                                     n0 * kBits / 8 + gi * p.y_gw, 0, p0, img);
+                }
+                bulk_commit();
+                bulk_wait_read<1>();
+                if (it > 0) mbar_arrive(&sfree[b ^ 1]);
+                trace_ev(p, 7, it);
+            }
+            bulk_wait<0>();
+        }
+    } else if (warp == kWarpTMA) {
         // ===================== TMA producer =====================
         if (lane == 0) {   // one thread issues (measured faster than an elected warp-wide loop)
             constexpr bool leader = true;
@@ -185,9 +212,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             tc_fence_after();
             const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
                                    static_cast<uint32_t>(buf * p.BN);
-            const bool storer = ew == 0 && lane == 0;
-            if (storer) bulk_wait_read<1>();
-            named_bar_sync(1, kNumEpiWarps * 32);
+            mbar_wait(&sfree[it & 1], (static_cast<uint32_t>(it >> 1) & 1u) ^ 1u);
             const uint32_t ystg_it = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes;
             // TMEM loads double-buffered: chunk ci+2 is in flight while chunk ci is requantized
             uint32_t va[32], vb[32];
@@ -229,20 +254,14 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 }
             }
             tc_fence_before();
+            fence_proxy_async_smem();                 // staging writes -> visible to the TMA store
             __syncwarp();
-            if (lane == 0) mbar_arrive(&tempty[buf]);
-            if (ew == 0 && lane == 0) trace_ev(p, 6, it);
-            fence_proxy_async_smem();
-            named_bar_sync(1, kNumEpiWarps * 32);
-            if (storer && !(p.exp_flags & 128)) {
-                constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
-                for (int gi = 0; gi < p.n_ygroups; ++gi)
-                    tma_store_4d(&ymap, smem + p.off_ystg + (it & 1) * p.ystg_bytes + gi * 128 * p.y_gw,
-                                 n0 * kBits / 8 + gi * p.y_gw, 0, p0, img);
-                bulk_commit();
+            if (lane == 0) {
+                mbar_arrive(&tempty[buf]);
+                mbar_arrive(&sfull[it & 1]);
             }
+            if (ew == 0 && lane == 0) trace_ev(p, 6, it);
         }
-        if (ew == 0 && lane == 0) bulk_wait<0>();
     } else if (IS4 && warp >= kWarpCvt0 && warp < kWarpCvt0 + kNumCvtWarps) {
         // ===================== int4 -> int8 plane widening =====================
         // packed plane j (16 B = 32 channels per pixel) -> int8 planes 2j (channels 0..15)

@@ -559,7 +559,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     if (p.n_mma > qc::kHaloMaxMMA) return false;
     p.off_mtab = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u, 16));
     p.off_bar = static_cast<uint32_t>(align_up(p.off_mtab + 8u * static_cast<uint32_t>(p.n_mma), 8));
-    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 5) * 8 + 16);
+    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 9) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
     if (pl->smem_bytes > 227u * 1024u) return false;
     p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), act_signed(d), dtype_signed(d->w_t));
