@@ -134,6 +134,7 @@ __device__ __forceinline__ void t_chan_mid(const ConvParams &p, TChan &c, int ne
 // 16 epilogue warps (4 per SMSP: the re-quantization is latency- not issue-bound), then the
 // 4 converter warps (4-bit).
 constexpr int kTEpiWarps = 16;
+constexpr int kTProducers = 2;        // TMA issuers: lane 0 of warps 0 and 3 (warp 2: output storer)
 constexpr int kTWarpCvt0 = kWarpEpi0 + kTEpiWarps;
 constexpr int kTThreads8 = 32 * kTWarpCvt0;
 constexpr int kTThreads4 = 32 * (kTWarpCvt0 + kNumCvtWarps);
@@ -189,11 +190,11 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
     const uint32_t tmem_base = *tmem_slot;
 
     if (warp == kWarpTMA || warp == 2 || warp == 3) {
-        // ===================== output storer (warp 2, lane 1) =====================
+        // ===================== output storer (warp 2, lane 0) =====================
         // The epilogue warps never wait for each other: each arrives on sfull[b] once its part
         // of staging buffer b is written; this thread waits for all 16, issues the TMA store, and
         // releases the other buffer (sfree) once the store issued before has read it.
-        if (warp == 2 && lane == 1) {
+        if (warp == 2 && lane == 0) {
             int it = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
                 const int b = it & 1;
@@ -210,9 +211,9 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             bulk_wait<0>();
         }
         // ===================== TMA producers =====================
-        if (lane == 0) {
+        if (lane == 0 && warp != 2) {   // lane 0 of warps 0 and 3 issue (warp 2 stores)
             griddep_wait();                                         // activations of the previous layer
-            const int pi = warp == kWarpTMA ? 0 : warp - 1;
+            const int pi = warp == kWarpTMA ? 0 : 1;
             const uint32_t tx = static_cast<uint32_t>(BNp * p.bkp + BMc * p.BK);
             int g = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
@@ -225,7 +226,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 const int wb = q0 * p.stride_w - p.pad_w;
                 const int hb = p0 * p.stride_h - p.pad_h;
                 for (int kb = 0; kb < p.num_kb; ++kb, ++g) {
-                    if (g % kNumProducers != pi) continue;
+                    if (g % kTProducers != pi) continue;
                     const int stage = g % NS;
                     const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
                     mbar_wait(&empty[stage], phase ^ 1u);
