@@ -17,7 +17,7 @@ from typing import Optional, Sequence, Tuple
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-_SO = os.environ.get("QC_LIBQCONV_DEBUG", os.path.join(_PKG, "libqconv.so"))   # debug override
+_SO = os.path.join(_PKG, "libqconv.so")
 
 QC_U4, QC_S4, QC_U8, QC_S8, QC_S32 = 0, 1, 2, 3, 4
 QC_F32, QC_BF16 = 0, 1
