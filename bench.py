@@ -518,6 +518,10 @@ def main():
     conv_bytes = np.array([L["bytes"] for L in trunk.layers], dtype=np.float64)
     conv_total_ms = float(conv_ms.sum())
     achieved_tops = conv_ops.sum() / (conv_total_ms / 1e3) / 1e12
+    # the layers whose arithmetic intensity is above the ridge point (tensor-bound on B200)
+    ridge = peaks["int8_tops_sustained"] * 1e12 / (peaks["hbm_gbs"] * 1e9)
+    cb = conv_ops / conv_bytes >= ridge
+    cb_tops = float(conv_ops[cb].sum() / (conv_ms[cb].sum() / 1e3) / 1e12) if cb.any() else None
     step_tops = trunk.ops_per_step / (ms_per_step / 1e3) / 1e12 * world / world
 
     e2e = None
@@ -561,6 +565,9 @@ def main():
                          "traffic_unit": "DRAM bytes per step over the 53 conv launches (ncu, profiles/)",
                          "peak_source": peaks["source"] + ", sustained",
                          "conv_share_of_step": conv_total_ms / instr_ms_per_step,
+                         "compute_bound_layers": {"count": int(cb.sum()), "ridge_ops_per_byte": ridge,
+                                                  "achieved": cb_tops,
+                                                  "frac": None if cb_tops is None else cb_tops / peaks["int8_tops_sustained"]},
                          "launch_times": "CUDA events after every launch, second pass of K instrumented "
                                          "graph replays right after the timed region",
                          "instrumented_ms_per_step": instr_ms_per_step,

@@ -204,9 +204,6 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
-            const int mt = tile / p.n_tiles_n;
-            const int img = mt / p.tiles_per_img;
-            const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
             mbar_wait(&tfull[buf], acc_phase);
             if (ew == 0 && lane == 0) trace_ev(p, 5, it);
             tc_fence_after();

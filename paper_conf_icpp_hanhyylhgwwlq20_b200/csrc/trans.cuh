@@ -312,7 +312,6 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
-            const int m0 = (tile / p.n_tiles_n) * kBNp;
             const int c0 = (tile % p.n_tiles_n) * BMc;
             if (c0 != cached_c0) {
                 const int ke = c0 + 2 * pair, ko = ke + 1;
