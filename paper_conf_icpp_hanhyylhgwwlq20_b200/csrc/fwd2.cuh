@@ -1,0 +1,317 @@
+// fwd2.cuh -- CTA-pair (cta_group::2) variant of the im2col implicit-GEMM conv.
+//
+// Same method as conv_fwd.cuh (Alg.2, fused epilogue P:L223/P:L253/P:L265); the
+// two CTAs of a cluster share one UMMA of M = 256 output pixels x N = BN output channels:
+// CTA r loads its 128 pixels of A and BN/2 rows of B per K-stage, the leader (rank 0) issues
+// `tcgen05.mma.cta_group::2`, and each CTA's TMEM receives its 128 rows of the accumulator.
+// Per CTA the shared-memory traffic per MAC drops by a third (B is split, not replicated),
+// which is what bounds the single-CTA kernel at N = 256.
+//
+// Cross-CTA protocol (all mbarriers live in each CTA at the same offsets):
+//   full[s]  (local)  : TMA landed (8-bit) / aready[s] (local): converter done (4-bit)
+//   peer[s]  (leader) : rank 1's stage s is ready -- rank 1's relay lane arrives remotely
+//   empty[s] (both)   : the pair's MMAs of stage s completed -- multicast commit
+//   tfull[b] (both)   : accumulator b complete -- multicast commit
+//   tempty[b](leader) : both CTAs' epilogue warps drained accumulator b -- local + remote arrives
+#pragma once
+#include "conv_fwd.cuh"
+
+namespace qc {
+
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t mapa_shared(uint32_t addr, uint32_t rank) {
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ void mbar_wait_cluster(uint64_t *bar, uint32_t parity) {
+    const uint32_t a = smem_u32(bar);
+    uint32_t ok = 0;
+    uint64_t t0 = 0;
+    uint32_t n = 0;
+    while (true) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(ok)
+            : "r"(a), "r"(parity)
+            : "memory");
+        if (ok) return;
+        if ((++n & 63u) == 0) {
+            const uint64_t t = globaltimer_ns();
+            if (t0 == 0) t0 = t;
+            else if (t - t0 > 4000000000ull) __trap();
+        }
+    }
+}
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+__device__ __forceinline__ void tmem_alloc2(uint32_t *dst_smem, uint32_t ncols) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
+                 "r"(ncols)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_dealloc2(uint32_t taddr, uint32_t ncols) {
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
+}
+__device__ __forceinline__ void mma2_i8_warp_lo(uint32_t d_tmem, uint32_t alo, uint32_t ahi, uint32_t blo,
+                                                uint32_t bhi, uint32_t idesc, uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p, e;\n\t.reg .b64 da, db;\n\t"
+        "setp.ne.b32 p, %6, 0;\n\t"
+        "mov.b64 da, {%1, %2};\n\t"
+        "mov.b64 db, {%3, %4};\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::2.kind::i8 [%0], da, db, %5, p;\n\t}" ::"r"(d_tmem),
+        "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "r"(accumulate)
+        : "memory");
+}
+// commit to the barrier at the same offset in both CTAs of the pair
+__device__ __forceinline__ void mma2_commit_mc_warp(uint64_t *bar) {
+    asm volatile(
+        "{\n\t.reg .pred e;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n\t}" ::"r"(
+            smem_u32(bar)),
+        "h"(static_cast<uint16_t>(3))
+        : "memory");
+}
+
+template <bool IS4, int OUT>
+__global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
+qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap wmap,
+                  const __grid_constant__ CUtensorMap ymap, const __grid_constant__ ConvParams p) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                                ~uintptr_t(1023));
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    const int NS = p.stages;
+    const uint32_t rank = cluster_ctarank();
+    const int pair = static_cast<int>(blockIdx.x >> 1), npairs = static_cast<int>(gridDim.x >> 1);
+    const int half_bn = p.BN / 2;
+
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + p.off_bar);
+    uint64_t *full = bars;                  // [NS]
+    uint64_t *empty = bars + NS;            // [NS]
+    uint64_t *aready = bars + 2 * NS;       // [NS]
+    uint64_t *peer = bars + 3 * NS;         // [NS] (leader)
+    uint64_t *tfull = bars + 4 * NS;        // [2]
+    uint64_t *tempty = bars + 4 * NS + 2;   // [2] (leader)
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 4 * NS + 4);
+    EpiCol *par = reinterpret_cast<EpiCol *>(smem + p.off_par);
+    int4 *chunk_info = reinterpret_cast<int4 *>(smem + p.off_par + 16 * kMaxBN);
+
+    griddep_launch_dependents();
+    if (warp == kWarpTMA && lane == 0) {
+        tma_prefetch_desc(&xmap);
+        tma_prefetch_desc(&wmap);
+        tma_prefetch_desc(&ymap);
+        for (int i = 0; i < NS; ++i) {
+            mbar_init(&full[i], 1);
+            mbar_init(&empty[i], 1);
+            mbar_init(&aready[i], kNumCvtWarps);
+            mbar_init(&peer[i], 1);
+        }
+        for (int i = 0; i < 2; ++i) {
+            mbar_init(&tfull[i], 1);
+            mbar_init(&tempty[i], 2 * kNumEpiWarps);
+        }
+        fence_mbar_init();
+    }
+    if (warp == kWarpMMA) tmem_alloc2(tmem_slot, p.tmem_cols);
+    tc_fence_before();
+    cluster_sync_all();                     // both CTAs' barriers initialised, TMEM allocated
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    const int taps_per_r = p.S * p.chunks;
+
+    if (warp == kWarpTMA || warp == 2 || warp == 3) {
+        // ===================== TMA producers: this CTA's A rows and B half =====================
+        if (lane == 0) {
+            griddep_wait();
+            const int pi = warp == kWarpTMA ? 0 : warp - 1;
+            const uint32_t tx = static_cast<uint32_t>(kBM * p.bkp + half_bn * p.BK);
+            int g = 0;
+            for (int tile = pair; tile < p.num_tiles; tile += npairs) {
+                const int m0 = (tile / p.n_tiles_n) * (2 * kBM) + static_cast<int>(rank) * kBM;
+                const int n0 = (tile % p.n_tiles_n) * p.BN + static_cast<int>(rank) * half_bn;
+                const int img = m0 / p.PQ;
+                const int rem = m0 - img * p.PQ;
+                const int p0 = rem / p.Q;
+                const int q0 = rem - p0 * p.Q;
+                const int wb = q0 * p.stride_w - p.pad_w;
+                const int hb = p0 * p.stride_h - p.pad_h;
+                for (int kb = 0; kb < p.num_kb; ++kb, ++g) {
+                    if (g % kNumProducers != pi) continue;
+                    const int stage = g % NS;
+                    const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
+                    mbar_wait(&empty[stage], phase ^ 1u);
+                    mbar_arrive_expect_tx(&full[stage], tx);
+                    const int r = kb / taps_per_r;
+                    const int rem2 = kb - r * taps_per_r;
+                    const int s = rem2 / p.chunks;
+                    const int ch = rem2 - s * p.chunks;
+                    uint8_t *adst = IS4 ? smem + p.off_stg + stage * p.stg_stage_bytes
+                                        : smem + p.off_a + stage * p.a_stage_bytes;
+                    tma_load_im2col_4d(adst, &xmap, &full[stage], ch * p.bkp, wb, hb, img,
+                                       static_cast<uint16_t>(s * p.dil_w), static_cast<uint16_t>(r * p.dil_h));
+                    tma_load_2d(smem + p.off_b + stage * p.b_stage_bytes, &wmap, &full[stage],
+                                (r * p.S + s) * p.C8 + ch * p.BK, n0);
+                }
+            }
+        }
+    } else if (warp == kWarpMMA) {
+        if (rank != 0) {
+            // ===================== relay (rank 1): my stage is ready -> leader =====================
+            if (lane == 0) {
+                const uint32_t peer0 = mapa_shared(smem_u32(peer), 0);
+                int g = 0;
+                for (int tile = pair; tile < p.num_tiles; tile += npairs) {
+                    for (int kb = 0; kb < p.num_kb; ++kb, ++g) {
+                        const int stage = g % NS;
+                        const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
+                        mbar_wait(IS4 ? &aready[stage] : &full[stage], phase);
+                        mbar_arrive_remote(peer0 + 8u * static_cast<uint32_t>(stage));
+                    }
+                }
+            }
+        } else {
+            // ===================== MMA issuer (leader, whole warp, one elected lane) =============
+            int stage = 0;
+            uint32_t phase = 0;
+            int it = 0;
+            const uint32_t sbo = 8u * static_cast<uint32_t>(p.BK);
+            const int ksteps = p.BK / 32;
+            for (int tile = pair; tile < p.num_tiles; tile += npairs, ++it) {
+                const int buf = it & 1;
+                const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
+                mbar_wait_cluster(&tempty[buf], acc_phase ^ 1u);
+                __syncwarp();
+                tc_fence_after();
+                const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
+                for (int kb = 0; kb < p.num_kb; ++kb) {
+                    mbar_wait(IS4 ? &aready[stage] : &full[stage], phase);
+                    mbar_wait_cluster(&peer[stage], phase);
+                    __syncwarp();
+                    tc_fence_after();
+                    const uint64_t ad0 = make_smem_desc(smem_u32(smem + p.off_a + stage * p.a_stage_bytes), 16u, sbo,
+                                                        p.sw_layout);
+                    const uint64_t bd0 = make_smem_desc(smem_u32(smem + p.off_b + stage * p.b_stage_bytes), 16u, sbo,
+                                                        p.sw_layout);
+                    const uint32_t alo = static_cast<uint32_t>(ad0), ahi = static_cast<uint32_t>(ad0 >> 32);
+                    const uint32_t blo = static_cast<uint32_t>(bd0), bhi = static_cast<uint32_t>(bd0 >> 32);
+                    for (int k = 0; k < ksteps; ++k)
+                        mma2_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
+                                        (kb | k) != 0 ? 1u : 0u);
+                    mma2_commit_mc_warp(&empty[stage]);
+                    if (++stage == NS) { stage = 0; phase ^= 1u; }
+                }
+                mma2_commit_mc_warp(&tfull[buf]);
+            }
+        }
+    } else if (warp >= kWarpEpi0 && warp < kWarpEpi0 + kNumEpiWarps) {
+        // ===================== epilogue: this CTA's 128 rows =====================
+        griddep_wait();
+        const int ew = warp - kWarpEpi0;
+        const int quarter = warp & 3;
+        const int half = ew >> 2;
+        const int row = quarter * 32 + lane;
+        const uint32_t par_base = smem_u32(par);
+        const int nchunks = (p.BN + 31) / 32;
+        const uint32_t tempty0 = mapa_shared(smem_u32(tempty), 0);
+        int cached_n0 = -1;
+        int it = 0;
+        const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
+        for (int tile = pair; tile < p.num_tiles; tile += npairs, ++it) {
+            const int buf = it & 1;
+            const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
+            const int m0 = (tile / p.n_tiles_n) * (2 * kBM) + static_cast<int>(rank) * kBM;
+            const int n0 = (tile % p.n_tiles_n) * p.BN;
+            if (n0 != cached_n0) {
+                fill_epilogue_params<OUT>(p, par, chunk_info, n0, ew, lane, false);
+                cached_n0 = n0;
+            }
+            mbar_wait(&tfull[buf], acc_phase);
+            tc_fence_after();
+            const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
+                                   static_cast<uint32_t>(buf * p.BN);
+            // one staging buffer (more room for the ring): the previous store must have read it
+            const bool storer = ew == 0 && lane == 0;
+            if (storer) bulk_wait_read<0>();
+            named_bar_sync(1, kNumEpiWarps * 32);
+            const uint32_t ystg_it = ystg_base;
+            for (int ci = half; ci < nchunks; ci += 2) {
+                uint32_t v[32];
+                __syncwarp();
+                tmem_ld_32x32b_x32(taddr + ci * 32, v);
+                tmem_wait_ld();
+                const int col0 = ci * 32;
+                const uint32_t pa = par_base + 16u * col0;
+                const int4 cinfo = chunk_info[ci];
+                epi_requant16<OUT, false, 0>(p, v, pa, cinfo, n0 + col0, 0, 0, 0, 0);
+                epi_requant16<OUT, false, 16>(p, v, pa, cinfo, n0 + col0, 0, 0, 0, 0);
+                stage16<OUT, 0>(p, v, ystg_it, row, col0);
+                stage16<OUT, 16>(p, v, ystg_it, row, col0 + 16);
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) {
+                if (rank == 0) mbar_arrive(&tempty[buf]);
+                else mbar_arrive_remote(tempty0 + 8u * static_cast<uint32_t>(buf));
+            }
+            fence_proxy_async_smem();
+            named_bar_sync(1, kNumEpiWarps * 32);
+            if (storer) {
+                constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
+                for (int g = 0; g < p.n_ygroups; ++g)
+                    tma_store_2d(&ymap, smem + p.off_ystg + g * 128 * p.y_gw,
+                                 n0 * kBits / 8 + g * p.y_gw, m0);
+                bulk_commit();
+            }
+        }
+        if (ew == 0 && lane == 0) bulk_wait<0>();
+    } else if (IS4 && warp >= kWarpCvt0 && warp < kWarpCvt0 + kNumCvtWarps) {
+        // ===================== int4 -> int8 widening of this CTA's A rows =====================
+        const int ct = (warp - kWarpCvt0) * 32 + lane;
+        const int cshift = p.cvt_shift;
+        const int nchunks = kBM << cshift;
+        const uint32_t xo = p.x_sgn4 ? 0x88888888u : 0u;
+        const uint32_t sw = static_cast<uint32_t>(p.sw_mask);
+        const uint32_t bkb = static_cast<uint32_t>(p.BK);
+        int stage = 0;
+        uint32_t phase = 0;
+        for (int tile = pair; tile < p.num_tiles; tile += npairs) {
+            for (int kb = 0; kb < p.num_kb; ++kb) {
+                mbar_wait(&full[stage], phase);
+                const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
+                const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
+                widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
+                fence_proxy_async_smem();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&aready[stage]);
+                if (++stage == NS) { stage = 0; phase ^= 1u; }
+            }
+        }
+    }
+
+    tc_fence_before();
+    cluster_sync_all();                     // nobody frees TMEM / exits while the pair is working
+    if (warp == kWarpMMA) {
+        __syncwarp();
+        tc_fence_after();
+        tmem_dealloc2(tmem_base, p.tmem_cols);
+    }
+}
+
+}  // namespace qc

@@ -21,6 +21,7 @@
 #include "prep.cuh"
 #include "halo.cuh"
 #include "trans.cuh"
+#include "fwd2.cuh"
 
 namespace {
 
@@ -466,6 +467,83 @@ qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &
                       const CUtensorMap &ym, cudaStream_t stream) {
     return pl.cp.x_zero != 0 ? launch_conv_t<IS4, OUT, true>(pl, xm, wm, ym, stream)
                              : launch_conv_t<IS4, OUT, false>(pl, xm, wm, ym, stream);
+}
+
+// ------------------------------------------------------------------ CTA-pair im2col (experimental)
+// QC_CTA2=1 routes the im2col layers that qualify to qconv_fwd2_kernel (fwd2.cuh).
+bool cta2_enabled() {
+    static const bool on = std::getenv("QC_CTA2") != nullptr;
+    return on;
+}
+
+bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, Plan *pl) {
+    if (!cta2_enabled()) return false;
+    if (pl1.cp.pair || d->x_zero != 0 || d->y_t == QC_S32 || !pl1.cp.y_tma) return false;
+    const int BN = pl1.BN;
+    if (BN % 32 || BN < 64) return false;
+    *pl = pl1;
+    qc::ConvParams &p = pl->cp;
+    const bool is4 = g.bits == 4;
+    const int m_tiles2 = static_cast<int>((g.M + 2 * qc::kBM - 1) / (2 * qc::kBM));
+    pl->num_tiles = m_tiles2 * pl1.n_tiles_n;
+    const uint32_t a_bytes = static_cast<uint32_t>(qc::kBM * pl1.BK);
+    const uint32_t b_bytes = static_cast<uint32_t>(align_up(static_cast<size_t>(BN / 2) * pl1.BK, 1024));
+    const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(qc::kBM * pl1.bkp) : 0u;
+    const uint32_t per_stage = a_bytes + b_bytes + stg_bytes;
+    const uint32_t ystg_bytes = p.ystg_bytes;                 // one staging buffer (fwd2.cuh)
+    const uint32_t fixed = static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 1024u + ystg_bytes;
+    int stages = static_cast<int>((227u * 1024u - 1024u - fixed) / per_stage);
+    stages = std::min(stages, 24);
+    if (stages < 2) return false;
+    pl->stages = stages;
+    p.stages = stages;
+    p.num_tiles = pl->num_tiles;
+    p.a_stage_bytes = a_bytes;
+    p.b_stage_bytes = b_bytes;
+    p.stg_stage_bytes = stg_bytes;
+    p.off_a = 0;
+    p.off_b = a_bytes * stages;
+    p.off_stg = p.off_b + b_bytes * stages;
+    p.off_ystg = static_cast<uint32_t>(align_up(p.off_stg + stg_bytes * stages, 1024));
+    p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + ystg_bytes, 16));
+    p.off_bar = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u, 8));
+    const uint32_t bar_bytes = static_cast<uint32_t>((4 * stages + 4) * 8 + 16);
+    pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
+    if (pl->smem_bytes > 227u * 1024u) return false;
+    p.idesc = qc::make_idesc_i8(2 * qc::kBM, static_cast<uint32_t>(BN), act_signed(d), dtype_signed(d->w_t));
+    const int pairs = std::min(pl->num_tiles, num_sms() / 2);
+    pl->grid = 2 * pairs;
+    return true;
+}
+
+template <bool IS4, int OUT>
+qc_status launch_fwd2(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm, const CUtensorMap &ym,
+                      cudaStream_t stream) {
+    auto kern = qc::qconv_fwd2_kernel<IS4, OUT>;
+    static int configured = 0;
+    if (!configured) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+        if (e != cudaSuccess) return cuda_fail(e);
+        configured = 1;
+    }
+    cudaLaunchConfig_t cfg;
+    std::memset(&cfg, 0, sizeof(cfg));
+    cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
+    cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
+    cfg.dynamicSmemBytes = pl.smem_bytes;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[2];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    qc::ConvParams cp = debug_params(pl.cp, stream);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
+    if (e != cudaSuccess) return cuda_fail(e);
+    debug_dump(cp, stream);
+    return QC_OK;
 }
 
 // ------------------------------------------------------------------ halo mode (stride 1)
@@ -1052,6 +1130,22 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
         if (s != QC_OK) return s;
     }
     const bool is4 = g.bits == 4;
+    {
+        Plan p2;
+        if (make_plan2(d, g, pl, &p2)) {
+            p2.cp.bias = bias; p2.cp.mult = multiplier; p2.cp.shift = shift; p2.cp.y = y;
+            alignas(64) CUtensorMap wm2;
+            s = encode_w_map(d, g, w8, pl.BK, pl.BN / 2, swizzle_for(pl.BK), &wm2);
+            if (s != QC_OK) return s;
+            switch (d->y_t) {
+                case QC_U8: return is4 ? launch_fwd2<true, qc::OUT_U8>(p2, xm, wm2, ym, st) : launch_fwd2<false, qc::OUT_U8>(p2, xm, wm2, ym, st);
+                case QC_S8: return is4 ? launch_fwd2<true, qc::OUT_S8>(p2, xm, wm2, ym, st) : launch_fwd2<false, qc::OUT_S8>(p2, xm, wm2, ym, st);
+                case QC_U4: return is4 ? launch_fwd2<true, qc::OUT_U4>(p2, xm, wm2, ym, st) : launch_fwd2<false, qc::OUT_U4>(p2, xm, wm2, ym, st);
+                case QC_S4: return is4 ? launch_fwd2<true, qc::OUT_S4>(p2, xm, wm2, ym, st) : launch_fwd2<false, qc::OUT_S4>(p2, xm, wm2, ym, st);
+                default: break;
+            }
+        }
+    }
     switch (d->y_t) {
         case QC_S32: return is4 ? launch_conv<true, qc::OUT_S32>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_S32>(pl, xm, wm, ym, st);
         case QC_U8: return is4 ? launch_conv<true, qc::OUT_U8>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_U8>(pl, xm, wm, ym, st);
