@@ -9,7 +9,8 @@
 //
 // Cross-CTA protocol (all mbarriers live in each CTA at the same offsets):
 //   full[s]  (local)  : TMA landed (8-bit) / aready[s] (local): converter done (4-bit)
-//   peer[s]  (leader) : rank 1's stage s is ready -- rank 1's relay lane arrives remotely
+//   8-bit: rank 1's TMA loads complete_tx on the LEADER's full[s] (.cta_group::2)
+//   4-bit: aready[s] (leader) counts both CTAs' converter warps (remote arrives from rank 1)
 //   empty[s] (both)   : the pair's MMAs of stage s completed -- multicast commit
 //   tfull[b] (both)   : accumulator b complete -- multicast commit
 //   tempty[b](leader) : both CTAs' epilogue warps drained accumulator b -- local + remote arrives
@@ -87,6 +88,24 @@ __device__ __forceinline__ void mma2_commit_mc_warp(uint64_t *bar) {
         : "memory");
 }
 
+// TMA loads into this CTA's shared memory that complete_tx on the LEADER's mbarrier
+// (`bar_cluster` = its shared::cluster address): .cta_group::2 lets the barrier be the peer's.
+__device__ __forceinline__ void tma2_load_2d(void *dst, const void *map, uint32_t bar_cluster, int32_t x, int32_t y) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.cta_group::2"
+        " [%0], [%1, {%3, %4}], [%2];" ::"r"(smem_u32(dst)),
+        "l"(map), "r"(bar_cluster), "r"(x), "r"(y)
+        : "memory");
+}
+__device__ __forceinline__ void tma2_load_im2col_4d(void *dst, const void *map, uint32_t bar_cluster, int32_t c,
+                                                    int32_t w, int32_t h, int32_t n, uint16_t off_w, uint16_t off_h) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes.cta_group::2"
+        " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(smem_u32(dst)),
+        "l"(map), "r"(bar_cluster), "r"(c), "r"(w), "r"(h), "r"(n), "h"(off_w), "h"(off_h)
+        : "memory");
+}
+
 template <bool IS4, int OUT>
 __global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
 qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap wmap,
@@ -120,7 +139,7 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
         for (int i = 0; i < NS; ++i) {
             mbar_init(&full[i], 1);
             mbar_init(&empty[i], 1);
-            mbar_init(&aready[i], kNumCvtWarps);
+            mbar_init(&aready[i], 2 * kNumCvtWarps);   // leader: both CTAs' converter warps
             mbar_init(&peer[i], 1);
         }
         for (int i = 0; i < 2; ++i) {
@@ -157,35 +176,36 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                     const int stage = g % NS;
                     const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
                     mbar_wait(&empty[stage], phase ^ 1u);
-                    mbar_arrive_expect_tx(&full[stage], tx);
                     const int r = kb / taps_per_r;
                     const int rem2 = kb - r * taps_per_r;
                     const int s = rem2 / p.chunks;
                     const int ch = rem2 - s * p.chunks;
                     uint8_t *adst = IS4 ? smem + p.off_stg + stage * p.stg_stage_bytes
                                         : smem + p.off_a + stage * p.a_stage_bytes;
-                    tma_load_im2col_4d(adst, &xmap, &full[stage], ch * p.bkp, wb, hb, img,
-                                       static_cast<uint16_t>(s * p.dil_w), static_cast<uint16_t>(r * p.dil_h));
-                    tma_load_2d(smem + p.off_b + stage * p.b_stage_bytes, &wmap, &full[stage],
-                                (r * p.S + s) * p.C8 + ch * p.BK, n0);
+                    if (IS4 || rank == 0) {
+                        // 4-bit: local barrier (the converter widens, the relay tells the leader);
+                        // 8-bit leader: the barrier also receives the peer's bytes
+                        mbar_arrive_expect_tx(&full[stage], (!IS4 ? 2u : 1u) * tx);
+                        tma_load_im2col_4d(adst, &xmap, &full[stage], ch * p.bkp, wb, hb, img,
+                                           static_cast<uint16_t>(s * p.dil_w), static_cast<uint16_t>(r * p.dil_h));
+                        tma_load_2d(smem + p.off_b + stage * p.b_stage_bytes, &wmap, &full[stage],
+                                    (r * p.S + s) * p.C8 + ch * p.BK, n0);
+                    } else {
+                        // 8-bit peer: its loads complete on the leader's barrier directly
+                        const uint32_t lb = mapa_shared(smem_u32(&full[stage]), 0);
+                        tma2_load_im2col_4d(adst, &xmap, lb, ch * p.bkp, wb, hb, img,
+                                            static_cast<uint16_t>(s * p.dil_w), static_cast<uint16_t>(r * p.dil_h));
+                        tma2_load_2d(smem + p.off_b + stage * p.b_stage_bytes, &wmap, lb,
+                                     (r * p.S + s) * p.C8 + ch * p.BK, n0);
+                    }
                 }
             }
         }
     } else if (warp == kWarpMMA) {
         if (rank != 0) {
-            // ===================== relay (rank 1): my stage is ready -> leader =====================
-            if (lane == 0) {
-                const uint32_t peer0 = mapa_shared(smem_u32(peer), 0);
-                int g = 0;
-                for (int tile = pair; tile < p.num_tiles; tile += npairs) {
-                    for (int kb = 0; kb < p.num_kb; ++kb, ++g) {
-                        const int stage = g % NS;
-                        const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
-                        mbar_wait(IS4 ? &aready[stage] : &full[stage], phase);
-                        mbar_arrive_remote(peer0 + 8u * static_cast<uint32_t>(stage));
-                    }
-                }
-            }
+            // the peer's stage readiness reaches the leader directly: its 8-bit TMA loads
+            // complete on the leader's `full`, its 4-bit converter warps arrive on the leader's
+            // `aready` -- the peer's MMA warp has nothing to do
         } else {
             // ===================== MMA issuer (leader, whole warp, one elected lane) =============
             int stage = 0;
@@ -201,8 +221,11 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
                 for (int kb = 0; kb < p.num_kb; ++kb) {
-                    mbar_wait(IS4 ? &aready[stage] : &full[stage], phase);
-                    mbar_wait_cluster(&peer[stage], phase);
+                    if (IS4) {
+                        mbar_wait_cluster(&aready[stage], phase);   // both CTAs' A widened
+                    } else {
+                        mbar_wait_cluster(&full[stage], phase);   // both CTAs' bytes landed
+                    }
                     __syncwarp();
                     tc_fence_after();
                     const uint64_t ad0 = make_smem_desc(smem_u32(smem + p.off_a + stage * p.a_stage_bytes), 16u, sbo,
@@ -289,6 +312,7 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
         const uint32_t xo = p.x_sgn4 ? 0x88888888u : 0u;
         const uint32_t sw = static_cast<uint32_t>(p.sw_mask);
         const uint32_t bkb = static_cast<uint32_t>(p.BK);
+        const uint32_t aready0 = mapa_shared(smem_u32(aready), 0);
         int stage = 0;
         uint32_t phase = 0;
         for (int tile = pair; tile < p.num_tiles; tile += npairs) {
@@ -299,7 +323,10 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                 widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
                 fence_proxy_async_smem();
                 __syncwarp();
-                if (lane == 0) mbar_arrive(&aready[stage]);
+                if (lane == 0) {
+                    if (rank == 0) mbar_arrive(&aready[stage]);
+                    else mbar_arrive_remote(aready0 + 8u * static_cast<uint32_t>(stage));
+                }
                 if (++stage == NS) { stage = 0; phase ^= 1u; }
             }
         }

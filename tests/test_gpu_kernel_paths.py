@@ -121,3 +121,35 @@ def test_int4_large_bias_general_mode(cs):
     m = rng.integers(1 << 30, 1 << 31, size=cs.k).astype(np.int32)
     n = rng.integers(40, 50, size=cs.k).astype(np.int32)
     _check(li, m, n)
+
+
+# ----------------------------------------------------------------------------- CTA-pair kernel
+@pytest.mark.parametrize("cs", [ConvShape("res4_3x3_b100", 100, 14, 14, 256, 256, 3, 3, 1, 1),
+                                ConvShape("res5_3x3_b400", 400, 7, 7, 512, 512, 3, 3, 1, 1)],
+                         ids=lambda c: c.name)
+def test_cta_pair_8bit_3x3_full_tiles(cs):
+    """8-bit 3x3 layers big enough for full N = 256 tiles take the CTA-pair kernel
+    (fwd2.cuh, cta_group::2): every output of three sampled images (first, last, one in
+    the middle -- each 256-pixel pair tile spans image boundaries) against the oracle."""
+    li = make_layer_inputs(cs, 8, seed=cs.n, relu=True)
+    m, n = oracle.requant_params(li.s_x, li.s_w, li.s_y)
+    got = _run(li, m, n)
+    for img in (0, cs.n // 2 + 1, cs.n - 1):
+        ref = oracle.conv2d_layer(li, mult=m, shift=n, n_slice=slice(img, img + 1))
+        np.testing.assert_array_equal(got[img:img + 1], ref, err_msg=f"{cs.name} img {img}")
+
+
+def test_cta_pair_forced_every_eligible_layer():
+    """QC_CTA2=1 (read once per process) forces the CTA-pair kernel onto every eligible
+    im2col layer, 4-bit included: run the small-shape and ResNet-50 parity tests that way in
+    a child process."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, QC_CTA2="1")
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu",
+                        os.path.join(root, "tests", "test_gpu_parity.py"), "-k",
+                        "small_shapes or resnet50_all or shift_ranges or signed_activations"],
+                       cwd=root, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
