@@ -53,8 +53,12 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t *bar, uint32_t parity
         }
     }
 }
+// Remote arrive with the default (.release.cta) semantics, as CUTLASS's ClusterBarrier does: a
+// .release.cluster arrive costs the converter warps ~0.5 us per stage (measured, trace_fwd2.py).
+// The data the leader's MMA then reads stays in this CTA's shared memory, made visible to the
+// async proxy by the preceding fence.proxy.async.
 __device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
-    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+    asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
 }
 __device__ __forceinline__ void tmem_alloc2(uint32_t *dst_smem, uint32_t ncols) {
     asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
@@ -104,6 +108,11 @@ __device__ __forceinline__ void tma2_load_im2col_4d(void *dst, const void *map, 
         " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(smem_u32(dst)),
         "l"(map), "r"(bar_cluster), "r"(c), "r"(w), "r"(h), "r"(n), "h"(off_w), "h"(off_h)
         : "memory");
+}
+
+// debug (QC_TRACE): events of CTA `cta` of the first pair
+__device__ __forceinline__ void trace_ev2(const ConvParams &p, int ev, int seq, uint32_t cta) {
+    if (p.trace != nullptr && blockIdx.x == cta && seq < 1024) p.trace[ev * 1024 + seq] = globaltimer_ns();
 }
 
 template <bool IS4, int OUT>
@@ -176,6 +185,7 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                     const int stage = g % NS;
                     const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
                     mbar_wait(&empty[stage], phase ^ 1u);
+                    trace_ev2(p, rank ? 7 : 0, g, rank);
                     const int r = kb / taps_per_r;
                     const int rem2 = kb - r * taps_per_r;
                     const int s = rem2 / p.chunks;
@@ -210,7 +220,7 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
             // ===================== MMA issuer (leader, whole warp, one elected lane) =============
             int stage = 0;
             uint32_t phase = 0;
-            int it = 0;
+            int it = 0, gs = 0;
             const uint32_t sbo = 8u * static_cast<uint32_t>(p.BK);
             const int ksteps = p.BK / 32;
             for (int tile = pair; tile < p.num_tiles; tile += npairs, ++it) {
@@ -221,6 +231,7 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
                 for (int kb = 0; kb < p.num_kb; ++kb) {
+                    trace_ev2(p, 2, gs, 0);
                     if (IS4) {
                         mbar_wait_cluster(&aready[stage], phase);   // both CTAs' A widened
                     } else {
@@ -238,6 +249,8 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                         mma2_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
                                         (kb | k) != 0 ? 1u : 0u);
                     mma2_commit_mc_warp(&empty[stage]);
+                    if (lane == 0) trace_ev2(p, 3, gs, 0);
+                    ++gs;
                     if (++stage == NS) { stage = 0; phase ^= 1u; }
                 }
                 mma2_commit_mc_warp(&tfull[buf]);
@@ -313,11 +326,13 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
         const uint32_t sw = static_cast<uint32_t>(p.sw_mask);
         const uint32_t bkb = static_cast<uint32_t>(p.BK);
         const uint32_t aready0 = mapa_shared(smem_u32(aready), 0);
+        int cg = 0;
         int stage = 0;
         uint32_t phase = 0;
         for (int tile = pair; tile < p.num_tiles; tile += npairs) {
             for (int kb = 0; kb < p.num_kb; ++kb) {
                 mbar_wait(&full[stage], phase);
+                if (ct == 0) trace_ev2(p, rank ? 8 : 5, cg, rank);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
                 widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
@@ -327,6 +342,8 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                     if (rank == 0) mbar_arrive(&aready[stage]);
                     else mbar_arrive_remote(aready0 + 8u * static_cast<uint32_t>(stage));
                 }
+                if (ct == 0) trace_ev2(p, rank ? 9 : 6, cg, rank);
+                ++cg;
                 if (++stage == NS) { stage = 0; phase ^= 1u; }
             }
         }

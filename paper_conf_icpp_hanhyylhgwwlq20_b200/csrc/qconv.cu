@@ -470,10 +470,10 @@ qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &
 }
 
 // ------------------------------------------------------------------ CTA-pair im2col (experimental)
-// The CTA-pair kernel (fwd2.cuh) runs 8-bit im2col layers with R*S > 1 and a full N = 256 tile
-// (measured faster there: res4/res5 3x3 -8 to -13 %; slower for narrower tiles and for 4-bit
-// inputs, whose cross-CTA converter hand-off is the bottleneck).  QC_CTA2=1 forces it for every
-// eligible layer (tests), QC_NO_CTA2=1 disables it.
+// The CTA-pair kernel (fwd2.cuh) runs im2col layers with R*S > 1 and a full N = 256 tile
+// (measured faster there: res4/res5 3x3 -6 to -13 % at 4 and 8 bits; no gain for 1x1 layers,
+// slower for N = 128 tiles).  QC_CTA2=1 forces it for every eligible layer (tests),
+// QC_NO_CTA2=1 disables it.
 bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, Plan *pl) {
     static const bool force = std::getenv("QC_CTA2") != nullptr;
     static const bool off = std::getenv("QC_NO_CTA2") != nullptr;
@@ -481,7 +481,7 @@ bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, Plan *p
     if (pl1.cp.pair || d->x_zero != 0 || d->y_t == QC_S32 || !pl1.cp.y_tma) return false;
     const int BN = pl1.BN;
     if (BN % 32 || BN < 64) return false;
-    if (!force && !(g.bits == 8 && BN == 256 && d->r * d->s > 1)) return false;
+    if (!force && !(BN == 256 && d->r * d->s > 1)) return false;
     *pl = pl1;
     qc::ConvParams &p = pl->cp;
     const bool is4 = g.bits == 4;
