@@ -558,7 +558,7 @@ def main():
                        "l2": "inputs > L2: 154 MB fp32 stem input and ~2.4 GB of trunk traffic per step",
                        "graph": "one CUDA graph per step (PDL between the conv kernels), replayed"},
             "tops": step_tops,
-            "roofline": {"bound": "tensor", "kernel": "the 53 conv launches (qconv_halo/qconv_t/qconv_fwd kernels)",
+            "roofline": {"bound": "tensor", "kernel": "the 53 conv launches (qconv_halo / qconv_t / qconv_fwd / qconv_fwd2 kernels)",
                          "achieved": achieved_tops, "peak": peaks["int8_tops_sustained"],
                          "unit": "TOPS", "frac": achieved_tops / peaks["int8_tops_sustained"],
                          "traffic": measured_traffic(args.bits, per_gpu),
