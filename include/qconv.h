@@ -133,8 +133,12 @@ size_t qconv2d_workspace_size(const qconv_desc *d);
  *                y = min(clamp_hi, max(clamp_lo, t + y_zero))     (Z3, Z5)
  * Contract (the paper's 32-bit accumulator): |acc| < 2^31 for
  * every output.  The host checks the dtype-range bound
- * r*s*c*max|x-x_zero|*max|w| < 2^31 (else OVERFLOW_RISK); keeping acc + bias
- * inside int32 is the caller's duty (bias is device data and is not read).
+ * r*s*c*max|x-x_zero|*max|w| < 2^31 (else OVERFLOW_RISK) -- for 4-bit inputs,
+ * whose on-chip widening accumulates 16x the sum, r*s*c*15*max|w| < 2^26 --
+ * and keeping acc + bias inside int32 is the caller's duty (bias is device data
+ * and is not read).  Every supported configuration gives the same bytes (the
+ * integer result is unique); which kernel runs (im2col, CTA-pair, halo,
+ * channel-major) is an internal choice.
  *   x          device, packed NHWC (d->x_t)
  *   w          device, packed KRSC (d->w_t) or prepared (d->w_prepared = 1)
  *   bias       device int32 [k] or NULL (= 0)
