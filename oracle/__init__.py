@@ -24,8 +24,9 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "oracle.c")
 
-U4, S4, U8, S8, S32 = 0, 1, 2, 3, 4
-_BITS = {U4: 4, S4: 4, U8: 8, S8: 8, S32: 32}
+U4, S4, U8, S8, S32, F32, BF16 = 0, 1, 2, 3, 4, 5, 6
+_BITS = {U4: 4, S4: 4, U8: 8, S8: 8, S32: 32, F32: 32, BF16: 16}
+ROUND_SINGLE, ROUND_TFLITE = 0, 1
 
 
 def build(force: bool = False) -> str:
@@ -53,6 +54,13 @@ def lib():
         L.oracle_conv2d.argtypes = [i32] * 7 + [i32] * 6 + [i32] * 3 + [i32, vp, i32, i32, i32] \
             + [vp, vp, vp, vp, vp, vp]
         L.oracle_conv2d.restype = i64
+        L.oracle_conv2d_ex.argtypes = [i32] * 7 + [i32] * 6 + [i32] * 3 + [i32, vp, i32, i32, i32, i32] \
+            + [vp, vp, vp, vp, vp, vp, i32, vp]
+        L.oracle_conv2d_ex.restype = i64
+        L.oracle_srdhm.argtypes = [ctypes.c_int32, ctypes.c_int32]
+        L.oracle_srdhm.restype = ctypes.c_int32
+        L.oracle_rdbpot.argtypes = [ctypes.c_int32, i32]
+        L.oracle_rdbpot.restype = ctypes.c_int32
         _lib = L
     return _lib
 
@@ -99,40 +107,59 @@ def conv_out_hw(h, w, r, s, stride_h, stride_w, pad_h, pad_w, dil_h, dil_w):
 def conv2d(x: np.ndarray, w: np.ndarray, *, n, h, wd, c, k, r, s, xt, wt, yt,
            stride=(1, 1), pad=(0, 0), dil=(1, 1), x_zero=0, w_zero=None, y_zero=0,
            clamp_lo=None, clamp_hi=None, bias=None, mult=None, shift=None,
+           rounding=ROUND_SINGLE, dq_scale=None, relu=False,
            allow_overflow=False) -> np.ndarray:
-    """Direct 7-loop quantized convolution (oracle.c:oracle_conv2d).
+    """Direct 7-loop quantized convolution (oracle.c:oracle_conv2d_ex).
 
     x, w: packed uint8 buffers (NHWC / KRSC).  Returns the packed output
-    buffer [n, p, q, k*bits/8] (uint8), or int32 [n,p,q,k] for yt == S32."""
+    buffer [n, p, q, k*bits/8] (uint8), int32 [n,p,q,k] for yt == S32, float32
+    [n,p,q,k] for yt == F32 and uint16 bf16 bit patterns [n,p,q,k] for BF16."""
     p, q = conv_out_hw(h, wd, r, s, stride[0], stride[1], pad[0], pad[1], dil[0], dil[1])
     x = np.ascontiguousarray(x, dtype=np.uint8)
     w = np.ascontiguousarray(w, dtype=np.uint8)
     if clamp_lo is None or clamp_hi is None:
-        lo = {U4: 0, S4: -8, U8: 0, S8: -128, S32: 0}[yt]
-        hi = {U4: 15, S4: 7, U8: 255, S8: 127, S32: 0}[yt]
+        lo = {U4: 0, S4: -8, U8: 0, S8: -128}.get(yt, 0)
+        hi = {U4: 15, S4: 7, U8: 255, S8: 127}.get(yt, 0)
         clamp_lo = lo if clamp_lo is None else clamp_lo
         clamp_hi = hi if clamp_hi is None else clamp_hi
     bias = None if bias is None else np.ascontiguousarray(bias, dtype=np.int32)
     mult = None if mult is None else np.ascontiguousarray(mult, dtype=np.int32)
     shift = None if shift is None else np.ascontiguousarray(shift, dtype=np.int32)
+    dqs = None if dq_scale is None else np.ascontiguousarray(dq_scale, dtype=np.float32)
     wz = None if w_zero is None else np.ascontiguousarray(w_zero, dtype=np.int32)
     if yt == S32:
         y = np.zeros((n, p, q, k), dtype=np.int32)
+    elif yt == F32:
+        y = np.zeros((n, p, q, k), dtype=np.float32)
+    elif yt == BF16:
+        y = np.zeros((n, p, q, k), dtype=np.uint16)
     else:
         y = np.zeros((n, p, q, k * _BITS[yt] // 8), dtype=np.uint8)
-    ov = lib().oracle_conv2d(n, h, wd, c, k, r, s, stride[0], stride[1], pad[0], pad[1],
-                             dil[0], dil[1], xt, wt, yt, int(x_zero), _ptr(wz), int(y_zero),
-                             int(clamp_lo), int(clamp_hi), _ptr(x), _ptr(w), _ptr(bias),
-                             _ptr(mult), _ptr(shift), _ptr(y))
+    ov = lib().oracle_conv2d_ex(n, h, wd, c, k, r, s, stride[0], stride[1], pad[0], pad[1],
+                                dil[0], dil[1], xt, wt, yt, int(x_zero), _ptr(wz), int(y_zero),
+                                int(clamp_lo), int(clamp_hi), int(rounding), _ptr(x), _ptr(w),
+                                _ptr(bias), _ptr(mult), _ptr(shift), _ptr(dqs), int(bool(relu)),
+                                _ptr(y))
     if ov < 0:
-        raise ValueError("oracle_conv2d: invalid arguments")
+        raise ValueError("oracle_conv2d_ex: invalid arguments")
     if ov > 0 and not allow_overflow:
         raise OverflowError(f"oracle_conv2d: {ov} accumulators outside int32 (outside the contract)")
     return y
 
 
-def conv2d_layer(li, mult=None, shift=None, y_t=None, bias=True, n_slice=None):
-    """Convenience: run the oracle on a workloads.LayerInputs (optionally a batch slice)."""
+def srdhm(a: int, b: int) -> int:
+    """gemmlowp SaturatingRoundingDoublingHighMul (oracle.c, reading Z15)."""
+    return int(lib().oracle_srdhm(int(a), int(b)))
+
+
+def rdbpot(x: int, e: int) -> int:
+    """gemmlowp RoundingDivideByPOT (oracle.c, reading Z15)."""
+    return int(lib().oracle_rdbpot(int(x), int(e)))
+
+
+def conv2d_layer(li, mult=None, shift=None, y_t=None, bias=True, n_slice=None, **kw):
+    """Convenience: run the oracle on a workloads.LayerInputs (optionally a batch slice);
+    extra keywords (rounding, dq_scale, relu, w_zero, ...) go to conv2d."""
     cs = li.shape
     yt = li.y_t if y_t is None else y_t
     c_st = li.x_codes.shape[-1]
@@ -145,4 +172,4 @@ def conv2d_layer(li, mult=None, shift=None, y_t=None, bias=True, n_slice=None):
                   xt=li.x_t, wt=li.w_t, yt=yt, stride=(cs.stride, cs.stride),
                   pad=(cs.pad, cs.pad), dil=(cs.dil, cs.dil), x_zero=li.x_zero, y_zero=li.y_zero,
                   clamp_lo=li.clamp_lo, clamp_hi=li.clamp_hi,
-                  bias=li.bias if bias else None, mult=mult, shift=shift)
+                  bias=li.bias if bias else None, mult=mult, shift=shift, **kw)

@@ -24,6 +24,19 @@
  *                            full reduction (Alg.2 l.15, P:L253,
  *                            reading Z11), ReLU by the truncation range
  *                            (reading Z5), int4/int8/int32 output.
+ *   oracle_conv2d_ex      -- the same convolution with the two NEXT epilogues
+ *                            of SURVEY 8 row f1/f3:
+ *                            * rounding = 1: gemmlowp/TFLite fixed-point
+ *                              re-quantization (reading Z15; "same
+ *                              quantization scheme", gemmlowp [14] P:L45):
+ *                              SaturatingRoundingDoublingHighMul then
+ *                              RoundingDivideByPOT, written as gemmlowp states
+ *                              them (oracle_srdhm / oracle_rdbpot)
+ *                            * yt = F32 / BF16: fusion of convolution and
+ *                              dequantization (section 4.4, reading
+ *                              Z16): y = fl32(fl32(acc) * scale[k]), acc incl.
+ *                              bias, optional ReLU y = (y > 0 ? y : +0), bf16 =
+ *                              round-to-nearest-even of the fp32 value.
  *
  * Parity pins: tests/test_oracle_pins.py (brute force, im2col+matmul,
  * 1x1==GEMM, identity/delta kernels, saturation, tie rule, requant params vs
@@ -35,9 +48,11 @@
 #include <string.h>
 
 /* dtype codes used by the oracle's own API (independent of include/qconv.h) */
-enum { OR_U4 = 0, OR_S4 = 1, OR_U8 = 2, OR_S8 = 3, OR_S32 = 4 };
+enum { OR_U4 = 0, OR_S4 = 1, OR_U8 = 2, OR_S8 = 3, OR_S32 = 4, OR_F32 = 5, OR_BF16 = 6 };
 
-static int dtype_bits(int t) { return (t == OR_U4 || t == OR_S4) ? 4 : (t == OR_S32 ? 32 : 8); }
+static int dtype_bits(int t) {
+    return (t == OR_U4 || t == OR_S4) ? 4 : ((t == OR_S32 || t == OR_F32) ? 32 : (t == OR_BF16 ? 16 : 8));
+}
 static int dtype_signed(int t) { return t == OR_S4 || t == OR_S8 || t == OR_S32; }
 static int64_t dtype_min(int t) {
     switch (t) { case OR_U4: return 0; case OR_S4: return -8; case OR_U8: return 0;
@@ -146,30 +161,81 @@ int oracle_requant_params(float in_scale, const float *w_scale, float out_scale,
 }
 
 /* ------------------------------------------------------------------------ */
-/* Direct convolution with the integer epilogue.
+/* gemmlowp fixed-point primitives (reading Z15), as gemmlowp defines them.
+ * SaturatingRoundingDoublingHighMul(a, b): the high 32 bits of 2*a*b with
+ * rounding: nudge = ab >= 0 ? 2^30 : 1 - 2^30, result = (ab + nudge) / 2^31
+ * with C's truncating division; the one overflowing case a = b = INT32_MIN
+ * saturates to INT32_MAX. */
+int32_t oracle_srdhm(int32_t a, int32_t b) {
+    if (a == INT32_MIN && b == INT32_MIN) return INT32_MAX;
+    const int64_t ab = (int64_t)a * (int64_t)b;
+    const int64_t nudge = ab >= 0 ? ((int64_t)1 << 30) : (1 - ((int64_t)1 << 30));
+    return (int32_t)((ab + nudge) / ((int64_t)1 << 31));
+}
+
+/* RoundingDivideByPOT(x, e): mask = 2^e - 1, remainder = x & mask,
+ * threshold = (mask >> 1) + (x < 0), result = (x >> e) + (remainder > threshold). */
+int32_t oracle_rdbpot(int32_t x, int e) {
+    const int32_t mask = (int32_t)(((int64_t)1 << e) - 1);
+    const int32_t remainder = x & mask;
+    const int32_t threshold = (mask >> 1) + (x < 0 ? 1 : 0);
+    return (x >> e) + (remainder > threshold ? 1 : 0);
+}
+
+/* TFLite MultiplyByQuantizedMultiplier with our (multiplier, shift) pair:
+ * the TFLite exponent is 31 - shift; a positive exponent is a left shift of
+ * the accumulator first (saturated to int32, reading Z15), a negative one the
+ * RoundingDivideByPOT after the high multiply. */
+static int64_t requant_tflite(int64_t acc, int32_t m, int sh) {
+    const int left = sh < 31 ? 31 - sh : 0;
+    const int right = sh > 31 ? sh - 31 : 0;
+    int64_t a = acc * ((int64_t)1 << left);
+    if (a > INT32_MAX) a = INT32_MAX;
+    if (a < INT32_MIN) a = INT32_MIN;
+    return oracle_rdbpot(oracle_srdhm((int32_t)a, m), right);
+}
+
+/* fp32 -> bf16 bit pattern, round to nearest even (finite inputs; the
+ * dequantized values are always finite). */
+static uint16_t f32_to_bf16_rne(float f) {
+    uint32_t u;
+    memcpy(&u, &f, 4);
+    const uint32_t lsb = (u >> 16) & 1u;
+    u += 0x7FFFu + lsb;
+    return (uint16_t)(u >> 16);
+}
+
+/* ------------------------------------------------------------------------ */
+/* Direct convolution with the integer or float epilogue.
  *
  * for n,p,q,k:
  *   acc = bias[k] + sum_{r,s in bounds} sum_c (X[n,h,w,c]-zx) * (W[k,r,s,c]-zw[k])
  *        (out-of-bounds taps are a real zero: they contribute nothing, Z2)
- *   S32 output: y = acc
- *   else      : t = floor((acc*m[k] + 2^(sh[k]-1)) / 2^sh[k])   (Z3, exact int128)
- *               y = min(hi, max(lo, t + zy))                      (Z5)
+ *   S32 output : y = acc
+ *   F32 / BF16 : y = fl32(fl32(acc) * dq_scale[k]); relu: y = y > 0 ? y : +0 (Z16)
+ *   else, rounding 0 : t = floor((acc*m[k] + 2^(sh[k]-1)) / 2^sh[k])   (Z3, exact int128)
+ *         rounding 1 : t = requant_tflite(acc, m[k], sh[k])            (Z15)
+ *               y = min(hi, max(lo, t + zy))                              (Z5)
  *
  * Returns the number of outputs whose acc lies outside int32 (the paper's
  * 32-bit accumulator: such an input is outside the method's
  * contract; the tests require 0).  Returns -1 on invalid arguments. */
-int64_t oracle_conv2d(int n_, int h_, int w_, int c_, int k_, int r_, int s_,
-                      int stride_h, int stride_w, int pad_h, int pad_w, int dil_h, int dil_w,
-                      int xt, int wt, int yt, int x_zero, const int32_t *w_zero,
-                      int y_zero, int clamp_lo, int clamp_hi,
-                      const uint8_t *x, const uint8_t *w, const int32_t *bias,
-                      const int32_t *mult, const int32_t *shift, uint8_t *y) {
+int64_t oracle_conv2d_ex(int n_, int h_, int w_, int c_, int k_, int r_, int s_,
+                         int stride_h, int stride_w, int pad_h, int pad_w, int dil_h, int dil_w,
+                         int xt, int wt, int yt, int x_zero, const int32_t *w_zero,
+                         int y_zero, int clamp_lo, int clamp_hi, int rounding,
+                         const uint8_t *x, const uint8_t *w, const int32_t *bias,
+                         const int32_t *mult, const int32_t *shift, const float *dq_scale,
+                         int relu, uint8_t *y) {
     if (n_ < 0 || h_ <= 0 || w_ <= 0 || c_ <= 0 || k_ <= 0 || r_ <= 0 || s_ <= 0) return -1;
     if (stride_h <= 0 || stride_w <= 0 || dil_h <= 0 || dil_w <= 0 || pad_h < 0 || pad_w < 0) return -1;
     const int P = (h_ + 2 * pad_h - dil_h * (r_ - 1) - 1) / stride_h + 1;
     const int Q = (w_ + 2 * pad_w - dil_w * (s_ - 1) - 1) / stride_w + 1;
     if (P <= 0 || Q <= 0) return -1;
-    if (yt != OR_S32 && (!mult || !shift)) return -1;
+    const int is_float = yt == OR_F32 || yt == OR_BF16;
+    if (is_float && !dq_scale) return -1;
+    if (!is_float && yt != OR_S32 && (!mult || !shift)) return -1;
+    if (rounding != 0 && rounding != 1) return -1;
     int64_t overflow = 0;
     #pragma omp parallel for collapse(2) schedule(static) reduction(+:overflow)
     for (int n = 0; n < n_; ++n) {
@@ -197,12 +263,28 @@ int64_t oracle_conv2d(int n_, int h_, int w_, int c_, int k_, int r_, int s_,
                     const int64_t oidx = (((int64_t)n * P + p) * Q + q) * k_ + k;
                     if (yt == OR_S32) {
                         put_elem(y, yt, oidx, acc);
+                    } else if (is_float) {
+                        volatile float fa = (float)acc;              /* RNE int -> fp32 */
+                        volatile float fy = fa * dq_scale[k];        /* one fp32 product */
+                        float v = fy;
+                        if (relu && !(v > 0.0f)) v = 0.0f;
+                        if (yt == OR_F32) {
+                            memcpy(y + 4 * oidx, &v, 4);
+                        } else {
+                            const uint16_t b = f32_to_bf16_rne(v);
+                            memcpy(y + 2 * oidx, &b, 2);
+                        }
                     } else {
                         const int sh = shift[k];
-                        __int128 prod = (__int128)acc * (__int128)mult[k];
-                        __int128 num = prod + ((__int128)1 << (sh - 1));
-                        /* floor division by 2^sh (arithmetic shift of int128 = floor) */
-                        __int128 t = num >> sh;
+                        __int128 t;
+                        if (rounding == 0) {
+                            __int128 prod = (__int128)acc * (__int128)mult[k];
+                            __int128 num = prod + ((__int128)1 << (sh - 1));
+                            /* floor division by 2^sh (arithmetic shift of int128 = floor) */
+                            t = num >> sh;
+                        } else {
+                            t = requant_tflite(acc, mult[k], sh);
+                        }
                         __int128 v = t + y_zero;
                         if (v < clamp_lo) v = clamp_lo;
                         if (v > clamp_hi) v = clamp_hi;
@@ -213,6 +295,19 @@ int64_t oracle_conv2d(int n_, int h_, int w_, int c_, int k_, int r_, int s_,
         }
     }
     return overflow;
+}
+
+/* The round-1 entry point: single rounding, integer outputs. */
+int64_t oracle_conv2d(int n_, int h_, int w_, int c_, int k_, int r_, int s_,
+                      int stride_h, int stride_w, int pad_h, int pad_w, int dil_h, int dil_w,
+                      int xt, int wt, int yt, int x_zero, const int32_t *w_zero,
+                      int y_zero, int clamp_lo, int clamp_hi,
+                      const uint8_t *x, const uint8_t *w, const int32_t *bias,
+                      const int32_t *mult, const int32_t *shift, uint8_t *y) {
+    if (yt == OR_F32 || yt == OR_BF16) return -1;
+    return oracle_conv2d_ex(n_, h_, w_, c_, k_, r_, s_, stride_h, stride_w, pad_h, pad_w, dil_h,
+                            dil_w, xt, wt, yt, x_zero, w_zero, y_zero, clamp_lo, clamp_hi, 0, x, w,
+                            bias, mult, shift, NULL, 0, y);
 }
 
 /* Smallest/largest representable values, exported for the Python wrapper. */

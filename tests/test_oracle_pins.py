@@ -367,3 +367,106 @@ def test_p1_exhaustive_tiny_4bit():
         got = unpack_codes(y, S8, 16)[0, 0]
         exp = np.array([[_round_half_up_exact(int(a) * int(b), m, n) for b in ws] for a in xs])
         np.testing.assert_array_equal(got, np.clip(exp, -128, 127))
+
+
+# ---------------------------------------------------------------------------- P13 (Z15)
+def _round_half_away_exact(fr: Fraction) -> int:
+    """Nearest integer, ties away from zero (what gemmlowp documents RoundingDivideByPOT to do)."""
+    a = abs(fr)
+    r = math.floor(a + Fraction(1, 2))
+    return r if fr >= 0 else -r
+
+
+def test_p13_gemmlowp_primitives_documented_values():
+    """Values fixed by gemmlowp's documentation of the two primitives (Q31 products, ties of
+    the divide away from zero) and the one saturating case."""
+    assert oracle.srdhm(1 << 30, 1 << 30) == 1 << 29            # 0.5 * 0.5 = 0.25 in Q31
+    assert oracle.srdhm(-(1 << 31), -(1 << 31)) == 2 ** 31 - 1  # saturation
+    assert oracle.srdhm(2 ** 31 - 1, 2 ** 31 - 1) == 2 ** 31 - 2
+    assert oracle.srdhm(-(1 << 31), 1 << 30) == -(1 << 30)
+    assert [oracle.rdbpot(v, 1) for v in (5, -5, 3, -3, 4, -4, 1, -1)] == [3, -3, 2, -2, 2, -2, 1, -1]
+    assert oracle.rdbpot(-(1 << 31), 31) == -1 and oracle.rdbpot(2 ** 31 - 1, 31) == 1
+    assert oracle.rdbpot(12345, 0) == 12345
+
+
+def test_p13_gemmlowp_primitives_vs_exact_rationals():
+    """SRDHM(a,b) = round-half-up(a*b / 2^31) and RDBPOT(x,e) = round-half-away(x / 2^e),
+    checked against exact rationals on random and tie-constructing operands."""
+    rng = np.random.default_rng(13)
+    lim = 2 ** 31
+    a = list(rng.integers(-lim, lim, 3000)) + [0, 1, -1, lim - 1, -lim, 1 << 30, -(1 << 30)]
+    b = list(rng.integers(-lim, lim, 3000)) + [lim - 1, lim - 1, lim - 1, 1, 1, 3, 3]
+    for x, y in zip(a, b):
+        x, y = int(x), int(y)
+        if x == -lim and y == -lim:
+            continue
+        exp = math.floor(Fraction(x * y, 2 ** 31) + Fraction(1, 2))
+        assert oracle.srdhm(x, y) == exp, (x, y)
+    for e in (0, 1, 2, 5, 13, 30, 31):
+        xs = list(rng.integers(-lim, lim, 300)) + [((2 * j + 1) << e) // 2 for j in range(-4, 4)
+                                                   if e > 0 and -lim <= ((2 * j + 1) << e) // 2 < lim]
+        for x in xs:
+            x = int(x)
+            assert oracle.rdbpot(x, e) == _round_half_away_exact(Fraction(x, 2 ** e)), (x, e)
+
+
+@pytest.mark.parametrize("m,sh", [(1 << 30, 31), (1518500250, 40), (1 << 30, 29), (2147483647, 62),
+                                  (1234567891, 35), (1 << 30, 1), (1 << 30, 33)])
+def test_p13_tflite_requant_through_conv(m, sh):
+    """rounding = 1 through the conv (acc = bias of a zero-input 1x1 conv): y = clamp(RDBPOT(
+    SRDHM(sat32(acc * 2^ls), m), rs)) with ls/rs from the TFLite exponent 31 - shift, each
+    step as an exact rational; and the single-rounding result differs on constructed ties."""
+    rng = np.random.default_rng(sh)
+    accs = np.array(list(rng.integers(-(2 ** 31), 2 ** 31, size=300)) + [0, 1, -1, 2 ** 31 - 1,
+                                                                        -(2 ** 31)], np.int64)
+    k = len(accs)
+    x = np.zeros((1, 1, 1, 32), dtype=np.int64)
+    w = np.zeros((k, 1, 1, 32), dtype=np.int64)
+    y = oracle.conv2d(pack_codes(x, U8), pack_codes(w, S8), n=1, h=1, wd=1, c=32, k=k, r=1, s=1,
+                      xt=U8, wt=S8, yt=S8, bias=accs.astype(np.int32), rounding=1,
+                      mult=np.full(k, m, np.int32), shift=np.full(k, sh, np.int32))
+    got = unpack_codes(y, S8, k)[0, 0, 0]
+    ls, rs = max(0, 31 - sh), max(0, sh - 31)
+    exp = []
+    for acc in accs:
+        a = min(2 ** 31 - 1, max(-(2 ** 31), int(acc) * 2 ** ls))
+        hm = math.floor(Fraction(a * m, 2 ** 31) + Fraction(1, 2))
+        exp.append(min(127, max(-128, _round_half_away_exact(Fraction(hm, 2 ** rs)))))
+    np.testing.assert_array_equal(got, np.array(exp))
+
+
+def test_p13_double_rounding_differs_from_single():
+    """acc*m/2^n = -2.5 exactly: single rounding (ties toward +inf) gives -2, the TFLite
+    double rounding (SRDHM exact here, RDBPOT ties away from zero) gives -3."""
+    m, sh = 1 << 30, 33                       # M = 2^-3: acc = -20 -> -2.5
+    x = np.zeros((1, 1, 1, 32), dtype=np.int64)
+    w = np.zeros((2, 1, 1, 32), dtype=np.int64)
+    kw = dict(n=1, h=1, wd=1, c=32, k=2, r=1, s=1, xt=U8, wt=S8, yt=S8,
+              bias=np.array([-20, 20], np.int32), mult=np.full(2, m, np.int32),
+              shift=np.full(2, sh, np.int32))
+    single = unpack_codes(oracle.conv2d(pack_codes(x, U8), pack_codes(w, S8), **kw), S8, 2)
+    tfl = unpack_codes(oracle.conv2d(pack_codes(x, U8), pack_codes(w, S8), rounding=1, **kw), S8, 2)
+    assert list(single[0, 0, 0]) == [-2, 3] and list(tfl[0, 0, 0]) == [-3, 3]
+
+
+# ---------------------------------------------------------------------------- P14 (Z16)
+@pytest.mark.parametrize("relu", [False, True])
+def test_p14_dequant_output_vs_numpy_and_torch(relu):
+    """Fusion of convolution and dequantization: y = fl32(fl32(acc) * scale[k]).
+    Checked against numpy's IEEE float32 product of the int32 result (a library routine, not
+    the oracle's own arithmetic) and, for bf16, torch's round-to-nearest-even conversion."""
+    from oracle import BF16, F32
+    li = make_layer_inputs(ConvShape("dq", 2, 9, 8, 32, 24, 3, 3, 1, 1), 8, seed=14, relu=False,
+                           signed_out=True)
+    li.bias[:4] = [2 ** 24 + 1, -(2 ** 24 + 3), 2 ** 30, -(2 ** 30)]   # int->fp32 rounding cases
+    acc = oracle.conv2d_layer(li, y_t=S32)
+    scale = (np.float32(li.s_x) * li.s_w).astype(np.float32)
+    ref = acc.astype(np.float32) * scale
+    if relu:
+        ref = np.where(ref > 0, ref, np.float32(0.0))
+    got = oracle.conv2d_layer(li, y_t=F32, dq_scale=scale, relu=relu)
+    assert got.dtype == np.float32
+    np.testing.assert_array_equal(got.view(np.uint32), ref.view(np.uint32))   # bit-exact, +0 only
+    gotb = oracle.conv2d_layer(li, y_t=BF16, dq_scale=scale, relu=relu)
+    refb = torch.from_numpy(ref).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
+    np.testing.assert_array_equal(gotb, refb)
