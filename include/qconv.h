@@ -48,8 +48,20 @@ typedef enum {
     QC_ERR_CUDA = 6            /* a CUDA driver/runtime call failed */
 } qc_status;
 
-typedef enum { QC_U4 = 0, QC_S4 = 1, QC_U8 = 2, QC_S8 = 3, QC_S32 = 4 } qc_dtype;
+/* QC_F32_OUT / QC_BF16_OUT: dequantized outputs of qconv2d_forward_dequant only. */
+typedef enum { QC_U4 = 0, QC_S4 = 1, QC_U8 = 2, QC_S8 = 3, QC_S32 = 4, QC_F32_OUT = 5,
+               QC_BF16_OUT = 6 } qc_dtype;
 typedef enum { QC_F32 = 0, QC_BF16 = 1 } qc_ftype;
+
+/* Re-quantization rounding (qconv_desc.rounding).
+ *  QC_ROUND_SINGLE (reading Z3): t = floor((acc*m + 2^(n-1)) / 2^n), one rounding, ties
+ *                   toward +inf.
+ *  QC_ROUND_TFLITE (reading Z15; the gemmlowp/TFLite scheme, "same quantization
+ *                   scheme", gemmlowp [14] P:L45): with ls = max(0, 31-n), rs = max(0, n-31),
+ *                   a = sat32(acc * 2^ls), h = SaturatingRoundingDoublingHighMul(a, m)
+ *                   = floor((a*m + 2^30) / 2^31) (INT32_MAX for a = m = INT32_MIN),
+ *                   t = RoundingDivideByPOT(h, rs) (nearest, ties away from zero). */
+typedef enum { QC_ROUND_SINGLE = 0, QC_ROUND_TFLITE = 1 } qc_rounding;
 
 /*
  * qconv_quantize_pack -- quantization step of the QNN layer sequence,
@@ -87,90 +99,172 @@ typedef struct {
     int32_t stride_h, stride_w;           /* 1..8 */
     int32_t pad_h, pad_w;                 /* >= 0 (zero padding = real zero, Z2) */
     int32_t dil_h, dil_w;                 /* >= 1 */
-    qc_dtype x_t, w_t, y_t;               /* x_t, w_t in {U4,S4,U8,S8}, same bit width;
-                                             y_t in {U4,S4,U8,S8,S32} */
+    qc_dtype x_t, w_t, y_t;               /* x_t, w_t in {U4,S4,U8,S8}: equal bit widths, or
+                                             8-bit activations with 4-bit weights (A8W4);
+                                             y_t in {U4,S4,U8,S8,S32} (qconv2d_forward) or
+                                             {F32_OUT,BF16_OUT} (qconv2d_forward_dequant) */
     int32_t x_zero;                       /* per-tensor activation zero point (Z1) */
+    const int32_t *w_zero;                /* device int32 [k] per-output-channel weight zero
+                                             points (Z1), or NULL (= 0).  Read by the device
+                                             only: any values inside the w_t range */
     int32_t w_prepared;                   /* 1: `w` is the output of qconv_prepare_weights */
-    int32_t y_zero;                       /* output zero point (ignored for S32) */
+    int32_t y_zero;                       /* output zero point (integer outputs except S32) */
     int32_t clamp_lo, clamp_hi;           /* truncation range inside the y_t range; ReLU:
                                              clamp_lo = max(qmin, y_zero) (Z5);
-                                             ignored for S32 */
+                                             ignored for S32 / float outputs */
+    int32_t rounding;                     /* qc_rounding (requantized outputs) */
+    int32_t relu;                         /* float outputs: y = (y > 0 ? y : +0) */
 } qconv_desc;
 
 /*
+ * Channel counts the kernels take directly: c % 32 == 0 (any width), or c == 16 at 8 bits
+ * (two filter taps per 32-byte K step).  Any other c is handled inside the library, with no
+ * change of the result (the same products, regrouped or padded with zero terms):
+ *  - stride 2, dilation 1 and 4*c <= 16 (the C = 3 / C = 4 image stems): the 2x2
+ *    space-to-depth form  X2[n,i,j,(2b+b')*c+cc] = x[n, 2i+b-pad_h, 2j+b'-pad_w, cc]
+ *    (x_zero outside), W2[k,a,a',(2b+b')*c+cc] = w[k, 2a+b, 2a'+b', cc] (0 beyond r, s):
+ *    a stride-1, unpadded ceil(r/2) x ceil(s/2) conv over 16 byte-coded channels;
+ *  - otherwise the channels are padded to 16 (8-bit, c < 16) or to a multiple of 32 with
+ *    x_zero activation codes and zero weights.
+ * The rearranged activations go to the workspace (qconv2d_workspace_size) on every call; the
+ * rearranged weights are what qconv_prepare_weights produces for such a descriptor.
+ */
+
+/*
  * qconv_prepare_weights -- once-per-layer weight preparation (the paper's
- * "pre-processing"): KRSC weights of dtype d->w_t are widened to the
+ * "pre-processing"): KRSC weights of dtype d->w_t are brought to the
  * kernel's operand layout (sm_100 tensor cores have no 4-bit integer MMA).
- * 8-bit weights are copied: k*r*s*c bytes.  4-bit weights (c % 32 == 0, else
- * UNSUPPORTED) become "nibble-plane" int8 KRSC -- within each 32-channel group
- * of a (k,r,s) row the 16 even channels come first as 16*w, then the 16 odd
- * channels as w, matching the kernel's on-chip activation widening -- followed,
- * 16-byte aligned, by int32 wsum[k] = sum over (r,s,c) of w (the correction of
- * signed 4-bit activations).  The layout is opaque to callers: only
- * qconv2d_forward (w_prepared = 1) reads it.
- * qconv_prepared_weight_bytes(d) = k*r*s*c (8-bit) or align16(k*r*s*c) + 4*k.
+ *  - 8-bit weights, c % 32 == 0 or c == 16: copied (k*r*s*c bytes).
+ *  - 4-bit weights with 4-bit activations: "nibble-plane" int8 KRSC -- within each
+ *    32-channel group of a (k,r,s) row the 16 even channels come first as 16*w, then the
+ *    16 odd channels as w, matching the kernel's on-chip activation widening -- followed,
+ *    16-byte aligned, by int32 wsum[k] = sum over (r,s,c) of w (the correction of signed
+ *    4-bit activations).
+ *  - 4-bit weights with 8-bit activations (A8W4): sign/zero-extended int8 KRSC.
+ *  - other channel counts: the space-to-depth or channel-padded weights (see above),
+ *    then as before.
+ * The layout is opaque to callers: only qconv2d_forward / qconv2d_forward_dequant with
+ * w_prepared = 1 read it.  qconv_prepared_weight_bytes(d) gives its size.
  *   w       device, packed KRSC (d->w_t)
  *   w_prep  device, >= qconv_prepared_weight_bytes(d) bytes
- * Errors: INVALID_ARG, MISALIGNED, CUDA.
+ * Errors: INVALID_ARG, UNSUPPORTED, MISALIGNED, CUDA.
  */
 size_t qconv_prepared_weight_bytes(const qconv_desc *d);
 qc_status qconv_prepare_weights(const qconv_desc *d, const void *w, void *w_prep, void *stream);
 
 /*
- * qconv2d_workspace_size -- device workspace bytes qconv2d_forward needs for
- * this descriptor: 0 unless x_zero != 0 (zero-point border table,
- * k*(r+1)*(s+1) int32) or 4-bit weights are passed unprepared (w_prepared = 0:
- * room for the prepared copy, qconv_prepared_weight_bytes(d) rounded up to 256).  Returns 0 for an invalid descriptor.
+ * qconv2d_workspace_size -- device workspace bytes qconv2d_forward needs for this
+ * descriptor (0 for the plain 4/8-bit layers of ResNet-50 / VGG with prepared or 8-bit
+ * weights).  Non-zero for: unprepared weights that need preparation (4-bit, A8W4, other
+ * channel counts), rearranged activations (c not taken directly, see above), x_zero != 0
+ * (zero-point border table, k*(r+1)*(s+1) int32) and w_zero != NULL (per-pixel activation
+ * sums).  Returns 0 for an invalid descriptor.
  */
 size_t qconv2d_workspace_size(const qconv_desc *d);
 
 /*
- * qconv2d_forward -- y = requant(conv(x - x_zero, w) + bias) (Alg.2).
+ * qconv2d_forward -- y = requant(conv(x - x_zero, w - w_zero) + bias) (Alg.2).
  * Per output (n,p,q,k), with acc = sum over in-bounds taps (r,s) and c of
- * (x[n, p*sh-ph+r*dh, q*sw-pw+s*dw, c] - x_zero) * w[k,r,s,c] + bias[k]:
+ * (x[n, p*sh-ph+r*dh, q*sw-pw+s*dw, c] - x_zero) * (w[k,r,s,c] - w_zero[k]) + bias[k]:
  *   y_t == S32 : y = acc
- *   otherwise  : t = floor((acc * multiplier[k] + 2^(shift[k]-1)) / 2^shift[k])
- *                y = min(clamp_hi, max(clamp_lo, t + y_zero))     (Z3, Z5)
- * Contract (the paper's 32-bit accumulator): |acc| < 2^31 for
- * every output.  The host checks the dtype-range bound
- * r*s*c*max|x-x_zero|*max|w| < 2^31 (else OVERFLOW_RISK) -- for 4-bit inputs,
- * whose on-chip widening accumulates 16x the sum, r*s*c*15*max|w| < 2^26 --
- * and keeping acc + bias inside int32 is the caller's duty (bias is device data
- * and is not read).  Every supported configuration gives the same bytes (the
- * integer result is unique); which kernel runs (im2col, CTA-pair, halo,
- * channel-major) is an internal choice.
+ *   otherwise  : t = rounding(acc, multiplier[k], shift[k])   (qc_rounding, Z3 / Z15)
+ *                y = min(clamp_hi, max(clamp_lo, t + y_zero))  (Z5)
+ * Domain of the per-channel device data: multiplier any int32 (qconv_requant_params gives
+ * [2^30, 2^31) or 0), shift in [1, 62]; a shift outside [1, 62] gives undefined bytes.
+ * Contract (the paper's 32-bit accumulator): |acc| < 2^31 for every output.
+ * The host checks the dtype-range bound r*s*c*max|x-x_zero|*max|w| < 2^31 (else
+ * OVERFLOW_RISK) -- for 4-bit activations, whose on-chip widening accumulates 16x the
+ * sum, r*s*c*15*max|w| < 2^26 -- and keeping acc + bias (and the w_zero terms) inside int32
+ * is the caller's duty (device data is not read on the host).  Every supported
+ * configuration gives the same bytes (the integer result is unique); which kernel runs
+ * (im2col, CTA-pair, halo, channel-major; see qconv_debug_plan) is an internal choice.
  *   x          device, packed NHWC (d->x_t)
  *   w          device, packed KRSC (d->w_t) or prepared (d->w_prepared = 1)
  *   bias       device int32 [k] or NULL (= 0)
  *   multiplier, shift   device int32 [k]; may be NULL only for y_t == S32
  *   y          device, NHWC [n,p,q,k] packed y_t
  *   workspace  device, >= qconv2d_workspace_size(d) bytes (NULL if 0)
- * Errors: INVALID_ARG, UNSUPPORTED (mixed bit widths; c not a multiple of 32 (8-bit
- * c = 16 is accepted: two filter taps per 32-byte K step);
- * 4-bit y_t with odd k; pad/dilation beyond the TMA im2col corner range;
- * stride > 8), OVERFLOW_RISK, MISALIGNED, WORKSPACE, CUDA.
+ * Errors: INVALID_ARG (also a float y_t: use qconv2d_forward_dequant), UNSUPPORTED
+ * (4-bit activations with 8-bit weights; 4-bit y_t with odd k; pad/dilation beyond the
+ * TMA im2col corner range; stride > 8), OVERFLOW_RISK, MISALIGNED, WORKSPACE, CUDA.
  */
 qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w,
                           const int32_t *bias, const int32_t *multiplier, const int32_t *shift,
                           void *y, void *workspace, size_t ws_bytes, void *stream);
 
 /*
- * Space-to-depth form of a stride-2 convolution (the ResNet/VGG C=3 stem).  For a
- * descriptor with stride 2 and dilation 1 (e.g. 7x7/s2/p3 over C=3), the 2x2
- * space-to-depth rearrangement
- *   X2[n,i,j,(2b+b')*c+cc] = code(x[n, 2i+b-pad_h, 2j+b'-pad_w, cc])  (x_zero where outside)
- *   W2[k,a,a',(2b+b')*c+cc] = w[k, 2a+b, 2a'+b', cc]                  (0 beyond r, s)
- * turns it into a stride-1, unpadded ceil(r/2) x ceil(s/2) convolution over C2 = 16
- * (4c <= 16) or round_up(4c, 32) channels whose output is identical, byte for byte, to
- * the original's (the same products, regrouped; P:L80's GEMM view with a denser K).
- * Codes are stored one per byte (4-bit codes sign/zero-extended) so C2 = 16 meets the
- * 16-byte TMA stride rule; the K reduction shrinks from r*s*round_up(c,32) to 16*C2.
+ * qconv2d_forward_dequant -- fusion of convolution and dequantization (section
+ * 4.4; reading Z16): the int32 result is converted to fp32 in the epilogue, with no
+ * integer store.  With acc as in qconv2d_forward (bias included):
+ *   y = fl32(fl32(acc) * scale[k])            (int32 -> fp32 and the product both RNE)
+ *   d->relu: y = (y > 0 ? y : +0)              (ReLU fusion)
+ *   d->y_t == QC_BF16_OUT: y rounded to bfloat16, nearest even.
+ *   scale   device float [k], normally fl32(s_x * s_w[k])
+ *   y       device, NHWC [n,p,q,k] fp32 or bf16
+ * Other arguments and errors as qconv2d_forward (y_t must be F32_OUT or BF16_OUT).
+ */
+qc_status qconv2d_forward_dequant(const qconv_desc *d, const void *x, const void *w,
+                                  const int32_t *bias, const float *scale, void *y,
+                                  void *workspace, size_t ws_bytes, void *stream);
+
+/*
+ * Launch plans and the per-shape tile search (the paper's "auto-search ... choose the
+ * best ones through profile runs", section 5.1).
+ *   kernel : QC_KERNEL_IM2COL   im2col implicit GEMM, one CTA per 128-pixel tile
+ *            QC_KERNEL_PAIR     im2col on a 2-CTA cluster (tcgen05 cta_group::2, M = 256)
+ *            QC_KERNEL_HALO     stride-1 halo tiles, weights resident in shared memory
+ *            QC_KERNEL_CHANNEL  1x1 convs, channel-major (output channels on TMEM lanes)
+ *   bn     : output channels per tile (IM2COL/PAIR: 16..256; CHANNEL: 64 or 128; HALO: K)
+ * qconv_debug_plan fills every field of the plan qconv2d_forward would launch for `d`
+ * (after any qconv_plan_set choice); the pre-kernels (weight preparation, activation
+ * rearrangement, zero-point tables) are listed in `prologue` as a bit mask
+ * (1 weights, 2 activations, 4 x_zero table, 8 w_zero sums).
+ * qconv_plan_set records a choice (kernel, bn; other fields ignored) for descriptors equal
+ * to `d` in every field (process-wide, thread-safe); an ineligible choice is rejected with
+ * UNSUPPORTED.  choice == NULL removes it.  qconv_plan_clear() removes all choices.
+ * qconv_plan_candidates writes up to `cap` eligible (kernel, bn) choices for `d` and
+ * returns how many exist.
+ * qconv_autotune times every candidate (`iters` launches each, CUDA events on `stream`,
+ * synchronous), records the fastest with qconv_plan_set and returns it in `best` and its
+ * mean time in `best_us`.  It writes `y` (every candidate gives the same bytes).
+ */
+typedef enum { QC_KERNEL_AUTO = 0, QC_KERNEL_IM2COL = 1, QC_KERNEL_PAIR = 2, QC_KERNEL_HALO = 3,
+               QC_KERNEL_CHANNEL = 4 } qc_kernel;
+typedef struct {
+    int32_t kernel;           /* qc_kernel */
+    int32_t bn;               /* output channels per tile */
+    int32_t bm;               /* output pixels per tile (per CTA pair for PAIR) */
+    int32_t stages;           /* shared-memory pipeline depth */
+    int32_t grid, threads;    /* launch shape (CTAs, threads per CTA) */
+    int32_t num_tiles;
+    int32_t smem_bytes, tmem_cols;
+    int32_t prologue;         /* pre-kernel mask, see above */
+    int32_t epilogue_mode;    /* 0 fast, 1 mid, 2 general: the mode all channels can take */
+    int32_t reserved[5];
+} qconv_plan;
+
+qc_status qconv_debug_plan(const qconv_desc *d, qconv_plan *out);
+qc_status qconv_plan_set(const qconv_desc *d, const qconv_plan *choice);
+void qconv_plan_clear(void);
+int32_t qconv_plan_candidates(const qconv_desc *d, qconv_plan *out, int32_t cap);
+qc_status qconv_autotune(const qconv_desc *d, const void *x, const void *w, const int32_t *bias,
+                         const int32_t *multiplier, const int32_t *shift, void *y,
+                         void *workspace, size_t ws_bytes, void *stream, int32_t iters,
+                         qconv_plan *best, float *best_us);
+
+/*
+ * Space-to-depth form of a stride-2 convolution (the ResNet/VGG C=3 stem), exposed so the
+ * fp32 quantization can write the rearranged codes directly.  qconv2d_forward applies the
+ * same rearrangement internally (above); these calls let the caller fuse it with the
+ * quantization step instead:
  *   qconv_s2d_desc          -> the transformed descriptor (x_t/w_t = byte containers,
  *                              w_prepared = 1); pass it to qconv2d_forward
  *   qconv_quantize_pack_s2d -> fused quantization (Z4, zero point d->x_zero, code range
  *                              of d->x_t) + rearrangement of fp32/bf16 NHWC x into X2
  *                              (device, qconv_s2d_desc(d).{n,h,w,c} bytes)
  *   qconv_prepare_weights_s2d -> W2 (device int8, qconv_prepared_weight_bytes_s2d bytes)
+ * Codes are stored one per byte (4-bit codes sign/zero-extended) so C2 = 16 meets the
+ * 16-byte TMA stride rule.
  * Errors: INVALID_ARG, UNSUPPORTED (stride != 2 or dilation != 1), MISALIGNED, CUDA.
  */
 qc_status qconv_s2d_desc(const qconv_desc *d, qconv_desc *out);

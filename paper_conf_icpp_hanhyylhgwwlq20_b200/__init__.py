@@ -19,9 +19,12 @@ import numpy as np
 _PKG = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_PKG, "libqconv.so")
 
-QC_U4, QC_S4, QC_U8, QC_S8, QC_S32 = 0, 1, 2, 3, 4
+QC_U4, QC_S4, QC_U8, QC_S8, QC_S32, QC_F32_OUT, QC_BF16_OUT = 0, 1, 2, 3, 4, 5, 6
 QC_F32, QC_BF16 = 0, 1
-_BITS = {QC_U4: 4, QC_S4: 4, QC_U8: 8, QC_S8: 8, QC_S32: 32}
+QC_ROUND_SINGLE, QC_ROUND_TFLITE = 0, 1
+QC_KERNEL_AUTO, QC_KERNEL_IM2COL, QC_KERNEL_PAIR, QC_KERNEL_HALO, QC_KERNEL_CHANNEL = 0, 1, 2, 3, 4
+KERNEL_NAMES = {0: "auto", 1: "im2col", 2: "pair", 3: "halo", 4: "channel"}
+_BITS = {QC_U4: 4, QC_S4: 4, QC_U8: 8, QC_S8: 8, QC_S32: 32, QC_F32_OUT: 32, QC_BF16_OUT: 16}
 _RANGE = {QC_U4: (0, 15), QC_S4: (-8, 7), QC_U8: (0, 255), QC_S8: (-128, 127),
           QC_S32: (-(2 ** 31), 2 ** 31 - 1)}
 
@@ -41,8 +44,21 @@ class QConvError(RuntimeError):
 class qconv_desc(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in
                 ("n", "h", "w", "c", "k", "r", "s", "stride_h", "stride_w", "pad_h", "pad_w",
-                 "dil_h", "dil_w", "x_t", "w_t", "y_t", "x_zero", "w_prepared", "y_zero",
-                 "clamp_lo", "clamp_hi")]
+                 "dil_h", "dil_w", "x_t", "w_t", "y_t", "x_zero")] + \
+               [("w_zero", ctypes.c_void_p)] + \
+               [(n, ctypes.c_int32) for n in ("w_prepared", "y_zero", "clamp_lo", "clamp_hi",
+                                               "rounding", "relu")]
+
+
+class qconv_plan(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in
+                ("kernel", "bn", "bm", "stages", "grid", "threads", "num_tiles", "smem_bytes",
+                 "tmem_cols", "prologue", "epilogue_mode")] + [("reserved", ctypes.c_int32 * 5)]
+
+    def as_dict(self):
+        d = {f: getattr(self, f) for f, _ in self._fields_ if f != "reserved"}
+        d["kernel_name"] = KERNEL_NAMES.get(self.kernel, str(self.kernel))
+        return d
 
 
 _L = None
@@ -74,6 +90,20 @@ def _lib():
         L.qconv2d_workspace_size.restype = sz
         L.qconv2d_forward.argtypes = [dp, vp, vp, vp, vp, vp, vp, vp, sz, vp]
         L.qconv2d_forward.restype = i32
+        L.qconv2d_forward_dequant.argtypes = [dp, vp, vp, vp, vp, vp, vp, sz, vp]
+        L.qconv2d_forward_dequant.restype = i32
+        pp = ctypes.POINTER(qconv_plan)
+        L.qconv_debug_plan.argtypes = [dp, pp]
+        L.qconv_debug_plan.restype = i32
+        L.qconv_plan_set.argtypes = [dp, pp]
+        L.qconv_plan_set.restype = i32
+        L.qconv_plan_clear.argtypes = []
+        L.qconv_plan_clear.restype = None
+        L.qconv_plan_candidates.argtypes = [dp, pp, i32]
+        L.qconv_plan_candidates.restype = i32
+        L.qconv_autotune.argtypes = [dp, vp, vp, vp, vp, vp, vp, vp, sz, vp, i32, pp,
+                                     ctypes.POINTER(ctypes.c_float)]
+        L.qconv_autotune.restype = i32
         L.qconv_s2d_desc.argtypes = [dp, dp]
         L.qconv_s2d_desc.restype = i32
         L.qconv_quantize_pack_s2d.argtypes = [dp, vp, i32, f32, vp, vp]
@@ -113,17 +143,23 @@ def _stream(stream) -> Optional[int]:
 # --------------------------------------------------------------------------- descriptors
 def make_desc(n, h, w, c, k, r, s, *, stride=1, pad=0, dil=1, x_t=QC_U8, w_t=QC_S8, y_t=QC_U8,
               x_zero=0, w_prepared=0, y_zero=0, clamp_lo=None, clamp_hi=None,
-              relu=False) -> qconv_desc:
+              relu=False, rounding=QC_ROUND_SINGLE, w_zero=None) -> qconv_desc:
+    """Descriptor (include/qconv.h).  w_zero: optional device int32 tensor [k] of weight zero
+    points -- the caller keeps it alive while the descriptor is used.  relu: for integer
+    outputs it narrows clamp_lo to max(qmin, y_zero); for float outputs it sets the
+    descriptor's relu flag."""
     sh, sw = (stride, stride) if isinstance(stride, int) else stride
     ph, pw = (pad, pad) if isinstance(pad, int) else pad
     dh, dw = (dil, dil) if isinstance(dil, int) else dil
-    lo, hi = _RANGE[y_t] if y_t != QC_S32 else (0, 0)
-    if relu and y_t != QC_S32:
+    packed = y_t in (QC_U4, QC_S4, QC_U8, QC_S8)
+    lo, hi = _RANGE[y_t] if packed else (0, 0)
+    if relu and packed:
         lo = max(lo, y_zero)
     lo = lo if clamp_lo is None else clamp_lo
     hi = hi if clamp_hi is None else clamp_hi
-    return qconv_desc(n, h, w, c, k, r, s, sh, sw, ph, pw, dh, dw, x_t, w_t, y_t, x_zero,
-                      w_prepared, y_zero, lo, hi)
+    wz = None if w_zero is None else (w_zero if isinstance(w_zero, int) else w_zero.data_ptr())
+    return qconv_desc(n, h, w, c, k, r, s, sh, sw, ph, pw, dh, dw, x_t, w_t, y_t, x_zero, wz,
+                      w_prepared, y_zero, lo, hi, rounding, 1 if (relu and not packed) else 0)
 
 
 def out_hw(d: qconv_desc) -> Tuple[int, int]:
@@ -189,23 +225,92 @@ def qconv2d_workspace_size(d: qconv_desc) -> int:
 
 def qconv2d_forward(d: qconv_desc, x, w, bias=None, multiplier=None, shift=None, y=None,
                     workspace=None, stream=None):
-    """y = requant(conv(x - x_zero, w) + bias) on the GPU (include/qconv.h)."""
-    import torch
+    """y = requant(conv(x - x_zero, w - w_zero) + bias) on the GPU (include/qconv.h)."""
     if y is None:
-        p, q = out_hw(d)
-        if d.y_t == QC_S32:
-            y = torch.empty((d.n, p, q, d.k), dtype=torch.int32, device=x.device)
-        else:
-            y = torch.empty((d.n, p, q, output_nbytes_per_pixel(d)), dtype=torch.uint8,
-                            device=x.device)
-    ws_need = qconv2d_workspace_size(d)
-    if ws_need and workspace is None:
-        workspace = torch.empty(ws_need, dtype=torch.uint8, device=x.device)
-    ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
+        y = _out_tensor(d, x.device)
+    workspace, ws_bytes = _workspace(d, workspace, x.device)
     _check("qconv2d_forward", _lib().qconv2d_forward(
         ctypes.byref(d), _ptr(x), _ptr(w), _ptr(bias), _ptr(multiplier), _ptr(shift), _ptr(y),
         _ptr(workspace), ws_bytes, _stream(stream)))
     return y
+
+
+def _out_tensor(d: qconv_desc, device):
+    import torch
+    p, q = out_hw(d)
+    if d.y_t == QC_S32:
+        return torch.empty((d.n, p, q, d.k), dtype=torch.int32, device=device)
+    if d.y_t == QC_F32_OUT:
+        return torch.empty((d.n, p, q, d.k), dtype=torch.float32, device=device)
+    if d.y_t == QC_BF16_OUT:
+        return torch.empty((d.n, p, q, d.k), dtype=torch.bfloat16, device=device)
+    return torch.empty((d.n, p, q, output_nbytes_per_pixel(d)), dtype=torch.uint8, device=device)
+
+
+def _workspace(d: qconv_desc, workspace, device):
+    import torch
+    ws_need = qconv2d_workspace_size(d)
+    if ws_need and workspace is None:
+        workspace = torch.empty(ws_need, dtype=torch.uint8, device=device)
+    ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
+    return workspace, ws_bytes
+
+
+def qconv2d_forward_dequant(d: qconv_desc, x, w, bias=None, scale=None, y=None, workspace=None,
+                            stream=None):
+    """y = fl32(fl32(conv(x - x_zero, w - w_zero) + bias) * scale[k]) (include/qconv.h, P:L263),
+    fp32 or bf16 per d.y_t."""
+    if y is None:
+        y = _out_tensor(d, x.device)
+    workspace, ws_bytes = _workspace(d, workspace, x.device)
+    _check("qconv2d_forward_dequant", _lib().qconv2d_forward_dequant(
+        ctypes.byref(d), _ptr(x), _ptr(w), _ptr(bias), _ptr(scale), _ptr(y), _ptr(workspace),
+        ws_bytes, _stream(stream)))
+    return y
+
+
+def qconv_debug_plan(d: qconv_desc) -> dict:
+    """The launch plan qconv2d_forward would use for `d` (kernel family, tiles, grid, ...)."""
+    p = qconv_plan()
+    _check("qconv_debug_plan", _lib().qconv_debug_plan(ctypes.byref(d), ctypes.byref(p)))
+    return p.as_dict()
+
+
+def qconv_plan_candidates(d: qconv_desc) -> list:
+    n = _lib().qconv_plan_candidates(ctypes.byref(d), None, 0)
+    arr = (qconv_plan * max(n, 1))()
+    _lib().qconv_plan_candidates(ctypes.byref(d), arr, n)
+    return [arr[i].as_dict() for i in range(n)]
+
+
+def qconv_plan_set(d: qconv_desc, kernel: Optional[int] = None, bn: int = 0):
+    """Record a (kernel, bn) choice for descriptors equal to `d`; kernel=None removes it."""
+    if kernel is None:
+        _check("qconv_plan_set", _lib().qconv_plan_set(ctypes.byref(d), None))
+        return
+    p = qconv_plan()
+    p.kernel, p.bn = int(kernel), int(bn)
+    _check("qconv_plan_set", _lib().qconv_plan_set(ctypes.byref(d), ctypes.byref(p)))
+
+
+def qconv_plan_clear():
+    _lib().qconv_plan_clear()
+
+
+def qconv_autotune(d: qconv_desc, x, w, bias=None, multiplier=None, shift=None, y=None,
+                   workspace=None, stream=None, iters: int = 10):
+    """Profile-run search over the eligible plans; records and returns the best
+    plan and its mean time in microseconds.  Synchronous."""
+    if y is None:
+        y = _out_tensor(d, x.device)
+    workspace, ws_bytes = _workspace(d, workspace, x.device)
+    best = qconv_plan()
+    us = ctypes.c_float()
+    _check("qconv_autotune", _lib().qconv_autotune(
+        ctypes.byref(d), _ptr(x), _ptr(w), _ptr(bias), _ptr(multiplier), _ptr(shift), _ptr(y),
+        _ptr(workspace), ws_bytes, _stream(stream), int(iters), ctypes.byref(best),
+        ctypes.byref(us)))
+    return best.as_dict(), float(us.value)
 
 
 def qconv_s2d_desc(d: qconv_desc) -> qconv_desc:
@@ -261,10 +366,11 @@ class QConv2d:
     multiplier: object
     shift: object
     workspace: object = None
+    scale: object = None          # float outputs: per-channel dequantization scale
 
     @classmethod
     def create(cls, desc: qconv_desc, w_bytes, bias, multiplier, shift, device="cuda",
-               stream=None):
+               stream=None, scale=None):
         import torch
         w_dev = torch.as_tensor(np.ascontiguousarray(w_bytes)).to(device)
         w_prep = qconv_prepare_weights(desc, w_dev, stream=stream)
@@ -275,14 +381,23 @@ class QConv2d:
         s = None if shift is None else torch.as_tensor(np.asarray(shift, np.int32)).to(device)
         ws = qconv2d_workspace_size(d)
         wsb = torch.empty(ws, dtype=torch.uint8, device=device) if ws else None
-        return cls(d, w_prep, b, m, s, wsb)
+        sc = None if scale is None else torch.as_tensor(np.asarray(scale, np.float32)).to(device)
+        return cls(d, w_prep, b, m, s, wsb, sc)
 
     def __call__(self, x, y=None, stream=None):
+        if self.desc.y_t in (QC_F32_OUT, QC_BF16_OUT):
+            return qconv2d_forward_dequant(self.desc, x, self.w_prep, self.bias, self.scale, y=y,
+                                           workspace=self.workspace, stream=stream)
         return qconv2d_forward(self.desc, x, self.w_prep, self.bias, self.multiplier, self.shift,
                                y=y, workspace=self.workspace, stream=stream)
 
 
 __all__ = ["qconv_quantize_pack", "qconv_requant_params", "qconv_prepare_weights",
+           "qconv2d_forward_dequant", "qconv_debug_plan", "qconv_plan_candidates",
+           "qconv_plan_set", "qconv_plan_clear", "qconv_autotune", "qconv_plan",
+           "QC_F32_OUT", "QC_BF16_OUT", "QC_ROUND_SINGLE", "QC_ROUND_TFLITE",
+           "QC_KERNEL_AUTO", "QC_KERNEL_IM2COL", "QC_KERNEL_PAIR", "QC_KERNEL_HALO",
+           "QC_KERNEL_CHANNEL",
            "qconv_s2d_desc", "qconv_quantize_pack_s2d", "qconv_prepare_weights_s2d",
            "qconv_prepared_weight_bytes", "qconv2d_workspace_size", "qconv2d_forward",
            "qconv_debug_im2col_tile", "make_desc", "qconv_desc", "QConv2d", "QConvError",

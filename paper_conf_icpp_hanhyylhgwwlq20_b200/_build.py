@@ -1,14 +1,20 @@
-"""Build libqconv.so in-tree with nvcc for sm_100a (no torch extension machinery)."""
+"""Build libqconv.so in-tree with nvcc for sm_100a (no torch extension machinery).
+
+Each csrc/*.cu translation unit (host ABI, and one per kernel family) is compiled to an
+object in parallel, then linked into one shared library with the CUDA runtime static."""
 from __future__ import annotations
 
 import glob
 import os
 import subprocess
+import sys
+from concurrent.futures import ThreadPoolExecutor
 
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 SO = os.path.join(PKG, "libqconv.so")
+OBJ = os.path.join(PKG, "build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 NVCC_FLAGS = [
@@ -16,13 +22,12 @@ NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=default",
     "--expt-relaxed-constexpr",
-    "-cudart", "static",
 ]
 
 
 def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cuh"))
-                  + [os.path.join(ROOT, "include", "qconv.h")])
+                  + glob.glob(os.path.join(CSRC, "*.h")) + [os.path.join(ROOT, "include", "qconv.h")])
 
 
 def needs_build() -> bool:
@@ -35,15 +40,32 @@ def needs_build() -> bool:
 def build(force: bool = False, verbose: bool = False, extra=()) -> str:
     if not force and not needs_build():
         return SO
-    cmd = [NVCC, *NVCC_FLAGS, *extra, "-I", os.path.join(ROOT, "include"), "-I", CSRC,
-           "-shared", "-o", SO + ".tmp", os.path.join(CSRC, "qconv.cu")]
+    os.makedirs(OBJ, exist_ok=True)
+    units = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
+
+    def compile_one(src):
+        obj = os.path.join(OBJ, os.path.basename(src)[:-3] + ".o")
+        cmd = [NVCC, *NVCC_FLAGS, *extra, *inc, "-c", "-o", obj, src]
+        if verbose:
+            print(" ".join(cmd), flush=True)
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError(f"nvcc failed on {src}:\n{r.stdout}\n{r.stderr}")
+        if verbose and r.stderr.strip():
+            print(r.stderr, file=sys.stderr)
+        return obj
+
+    with ThreadPoolExecutor(max_workers=min(len(units), os.cpu_count() or 4)) as ex:
+        objs = list(ex.map(compile_one, units))
+    cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-cudart", "static", "-shared",
+           "-o", SO + ".tmp", *objs]
     if verbose:
-        print(" ".join(cmd))
+        print(" ".join(cmd), flush=True)
     subprocess.check_call(cmd)
     os.replace(SO + ".tmp", SO)
     return SO
 
 
 if __name__ == "__main__":
-    import sys
     build(force=True, verbose=True, extra=sys.argv[1:])

@@ -15,7 +15,7 @@
 //   tfull[b] (both)   : accumulator b complete -- multicast commit
 //   tempty[b](leader) : both CTAs' epilogue warps drained accumulator b -- local + remote arrives
 #pragma once
-#include "conv_fwd.cuh"
+#include "epilogue.cuh"
 
 namespace qc {
 
@@ -111,9 +111,13 @@ __device__ __forceinline__ void tma2_load_im2col_4d(void *dst, const void *map, 
 }
 
 // debug (QC_TRACE): events of CTA `cta` of the first pair
+#ifdef QC_DEBUG
 __device__ __forceinline__ void trace_ev2(const ConvParams &p, int ev, int seq, uint32_t cta) {
     if (p.trace != nullptr && blockIdx.x == cta && seq < 1024) p.trace[ev * 1024 + seq] = globaltimer_ns();
 }
+#else
+__device__ __forceinline__ void trace_ev2(const ConvParams &, int, int, uint32_t) {}
+#endif
 
 template <bool IS4, int OUT>
 __global__ void __launch_bounds__(IS4 ? 512 : 384, 1)

@@ -17,11 +17,10 @@
 // The paper's precomputed-offset gather and register prefetch
 // have no counterpart: the hardware gathers, shared memory reuses.
 #pragma once
-#include "conv_fwd.cuh"
+#include "epilogue.cuh"
 
 namespace qc {
 
-constexpr int kHaloMaxMMA = 18;      // 3x3 taps x 2 plane pairs (C = 64), or the 4x4/2 stem pairs
 
 template <bool IS4, int OUT>
 __global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
@@ -84,7 +83,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 const int img = mt / p.tiles_per_img;
                 const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
                 mbar_wait(&sfull[b], static_cast<uint32_t>(it >> 1) & 1u);
-                if (!(p.exp_flags & 128)) {
+                {
                     constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
                     for (int gi = 0; gi < p.n_ygroups; ++gi)
                         tma_store_4d(&ymap, smem + p.off_ystg + b * p.ystg_bytes + gi * 128 * p.y_gw,
@@ -101,10 +100,11 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         // ===================== TMA producer =====================
         if (lane == 0) {   // one thread issues (measured faster than an elected warp-wide loop)
             constexpr bool leader = true;
-            if (!p.w_early) griddep_wait();                         // weights prepared in this call
+            // the weights may have been written by the kernel just before this one in the
+            // stream (weight preparation, or the caller's own kernels): wait for it first
+            griddep_wait();
             if (leader) mbar_arrive_expect_tx(bfull, p.b_res_bytes);
             if (leader) tma_load_3d(smem + p.off_bres, &bmap, bfull, 0, n0, 0);
-            if (p.w_early) griddep_wait();                          // activations of the previous layer
             int g = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
                 const int mt = tile / p.n_tiles_n;
@@ -175,7 +175,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 // fully unrolled over the precomputed per-MMA offsets (registers)
 #pragma unroll
                 for (int i = 0; i < kHaloMaxMMA; ++i) {
-                    if (i < nmma && (!(p.exp_flags & 4) || i == 0) && !(p.exp_flags & 64))   // debug ablations
+                    if (i < nmma)
                         mma_i8_warp_lo(d_tmem, alo0 + aoff[i], ahi, blo0 + boff[i], bhi, p.idesc, i > 0 ? 1u : 0u);
                 }
                 if (leader) trace_ev(p, 11, it);
@@ -215,10 +215,6 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             uint32_t va[32], vb[32];
             auto process = [&](uint32_t (&v)[32], int ci) {
                 const int col0 = ci * 32;
-                if (p.exp_flags & 16) {            // debug ablation: TMEM loads only
-                    if (v[0] == 0x9e3779b9u && col0 == 12345) asm volatile("trap;");
-                    return;
-                }
                 const uint32_t pa = par_base + 16u * col0;
                 const int4 cinfo = chunk_info[ci];
                 epi_requant16<OUT, false, 0>(p, v, pa, cinfo, n0 + col0, 0, 0, 0, 0);

@@ -1,11 +1,18 @@
 // prep.cuh -- memory-bound kernels around the convolution:
 //   quantize_pack_kernel : fp32/bf16 NHWC -> packed int8/int4 NHWC (Z4)
 //   widen_w4_kernel      : packed int4 KRSC weights -> nibble-plane int8 KRSC (once per layer)
+//   widen_w4_pad_kernel  : the same with channel padding (c not a multiple of 32)
 //   wsum_w4_kernel       : per-channel weight sums (signed 4-bit activation offset)
+//   weights_plain_kernel : 4/8-bit KRSC -> int8 KRSC with channel padding (A8W4, 8-bit padding)
+//   repack_pad_kernel    : activation codes with channels padded by x_zero codes
+//   repack_s2d_kernel    : activation codes -> 2x2 space-to-depth byte codes (stride-2 stems)
 //   zx_table_kernel      : 2-D prefix sums of sum_c w[k,r,s,c] for x_zero != 0 borders (Z2)
+//   chsum_kernel, x1_kernel : per-output-pixel sums of (x - x_zero) over in-bounds taps, the
+//                          correction term of per-channel weight zero points (Z1)
 #pragma once
 #include <cstdint>
 #include <cuda_bf16.h>
+#include "ptx.cuh"
 
 namespace qc {
 
@@ -258,49 +265,143 @@ __global__ void __launch_bounds__(256) quantize_s2d_kernel(const __grid_constant
     }
 }
 
-// Row-blocked variant for 4c <= 16 and w*c <= 4096: one CTA per (image, output row i)
-// stages the two input rows 2i-pad_h, 2i+1-pad_h in shared memory with coalesced 16-byte
-// loads, then thread j emits the 16 codes of X2[n, i, j, :] as one 16-byte store.
-__global__ void __launch_bounds__(128) quantize_s2d_rows_kernel(const __grid_constant__ QuantS2DParams p) {
-    __shared__ __align__(16) float rows[2][4096];
-    QuantParams qp;
-    qp.x = p.x; qp.inv_s = p.inv_s; qp.flo = p.flo; qp.fhi = p.fhi;
-    qp.z = p.z; qp.qmin = p.qmin; qp.qmax = p.qmax; qp.bf16 = p.bf16;
-    const int32_t rowlen = p.w * p.c;
-    for (int64_t blk = blockIdx.x; blk < static_cast<int64_t>(p.n) * p.hs; blk += gridDim.x) {
-        const int64_t img = blk / p.hs;
-        const int32_t i = static_cast<int32_t>(blk - img * p.hs);
-        __syncthreads();
-        for (int b = 0; b < 2; ++b) {
-            const int32_t hh = 2 * i + b - p.pad_h;
-            if (hh < 0 || hh >= p.h) continue;
-            const int64_t base = (img * p.h + hh) * rowlen;
-            if (!p.bf16 && (rowlen % 4) == 0) {
-                const float4 *src = reinterpret_cast<const float4 *>(static_cast<const float *>(p.x) + base);
-                for (int t = threadIdx.x; t < rowlen / 4; t += blockDim.x)
-                    reinterpret_cast<float4 *>(rows[b])[t] = __ldg(src + t);
-            } else {
-                for (int t = threadIdx.x; t < rowlen; t += blockDim.x) rows[b][t] = load_x(qp, base + t);
+// Code of element `idx` of a packed row-major 4/8-bit buffer (Z7 nibble order), as int.
+__device__ __forceinline__ int32_t get_code(const uint8_t *__restrict__ buf, int64_t idx, int32_t bits,
+                                            int32_t is_signed) {
+    if (bits == 8) return is_signed ? static_cast<int32_t>(static_cast<int8_t>(buf[idx])) : static_cast<int32_t>(buf[idx]);
+    const uint8_t b = buf[idx >> 1];
+    int32_t v = (idx & 1) ? (b >> 4) : (b & 0xF);
+    if (is_signed && v >= 8) v -= 16;
+    return v;
+}
+
+// Nibble-plane prepared weights (widen_w4_kernel's layout) of 4-bit KRSC weights whose rows
+// of c_src channels are padded with zero weights to c_dst (a multiple of 32) channels.
+__global__ void __launch_bounds__(256) widen_w4_pad_kernel(const uint8_t *__restrict__ w4,
+                                                           int8_t *__restrict__ w8, int64_t rows,
+                                                           int32_t c_src, int32_t c_dst, int32_t is_signed) {
+    const int32_t gpr = c_dst / 32;
+    const int64_t n_groups = rows * gpr;
+    for (int64_t i = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; i < n_groups;
+         i += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t row = i / gpr;
+        const int32_t c0 = static_cast<int32_t>(i - row * gpr) * 32;
+        int8_t *dst = w8 + row * c_dst + c0;
+        for (int p = 0; p < 16; ++p) {
+            const int32_t ce = c0 + 2 * p, co = ce + 1;
+            const int32_t e = ce < c_src ? get_code(w4, row * c_src + ce, 4, is_signed) : 0;
+            const int32_t o = co < c_src ? get_code(w4, row * c_src + co, 4, is_signed) : 0;
+            dst[p] = static_cast<int8_t>(16 * e);
+            dst[16 + p] = static_cast<int8_t>(o);
+        }
+    }
+}
+
+// int8 KRSC from 4- or 8-bit packed KRSC, rows of c_src channels padded to c_dst with zero
+// weights (A8W4 weights; 8-bit channel padding).
+__global__ void __launch_bounds__(256) weights_plain_kernel(const uint8_t *__restrict__ w, int8_t *__restrict__ w8,
+                                                            int64_t rows, int32_t c_src, int32_t c_dst,
+                                                            int32_t bits, int32_t is_signed) {
+    const int64_t total = rows * c_dst;
+    for (int64_t e = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; e < total;
+         e += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t row = e / c_dst;
+        const int32_t c = static_cast<int32_t>(e - row * c_dst);
+        w8[e] = static_cast<int8_t>(c < c_src ? get_code(w, row * c_src + c, bits, is_signed) : 0);
+    }
+}
+
+// Activation codes [npix][c_src] -> [npix][c_dst] (same packing), pad channels = zx.
+__global__ void __launch_bounds__(256) repack_pad_kernel(const uint8_t *__restrict__ x, uint8_t *__restrict__ y,
+                                                         int64_t npix, int32_t c_src, int32_t c_dst,
+                                                         int32_t bits, int32_t zx) {
+    const int32_t ob = c_dst * bits / 8;      // output bytes per pixel
+    const int64_t total = npix * ob;
+    for (int64_t e = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; e < total;
+         e += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t pix = e / ob;
+        const int32_t j = static_cast<int32_t>(e - pix * ob);
+        if (bits == 8) {
+            y[e] = j < c_src ? x[pix * c_src + j] : static_cast<uint8_t>(zx & 0xFF);
+        } else {
+            uint32_t v = 0;
+            for (int h = 0; h < 2; ++h) {
+                const int32_t c = 2 * j + h;
+                const int64_t idx = pix * c_src + c;
+                const uint32_t nib = c < c_src ? ((x[idx >> 1] >> (4 * (idx & 1))) & 0xFu) : (static_cast<uint32_t>(zx) & 0xFu);
+                v |= nib << (4 * h);
+            }
+            y[e] = static_cast<uint8_t>(v);
+        }
+    }
+}
+
+// Activation codes (4/8-bit packed, c channels) -> space-to-depth byte codes X2 [n][hs][ws][cs]:
+// X2[n,i,j,(2b+b')*c+cc] = code(x[n, 2i+b-pad_h, 2j+b'-pad_w, cc]), zx outside the image or
+// beyond 4c; 4-bit codes sign/zero-extended to a byte.
+__global__ void __launch_bounds__(256) repack_s2d_kernel(const uint8_t *__restrict__ x, uint8_t *__restrict__ y,
+                                                         int32_t n, int32_t h, int32_t w, int32_t c,
+                                                         int32_t hs, int32_t ws, int32_t cs, int32_t pad_h,
+                                                         int32_t pad_w, int32_t bits, int32_t is_signed,
+                                                         int32_t zx) {
+    const int64_t total = static_cast<int64_t>(n) * hs * ws * cs;
+    for (int64_t e = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; e < total;
+         e += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        int64_t rest = e;
+        const int32_t ch = static_cast<int32_t>(rest % cs); rest /= cs;
+        const int32_t j = static_cast<int32_t>(rest % ws); rest /= ws;
+        const int32_t i = static_cast<int32_t>(rest % hs); rest /= hs;
+        const int64_t img = rest;
+        int32_t code = zx;
+        if (ch < 4 * c) {
+            const int32_t blk = ch / c, cc = ch - blk * c;
+            const int32_t hh = 2 * i + (blk >> 1) - pad_h;
+            const int32_t ww = 2 * j + (blk & 1) - pad_w;
+            if (hh >= 0 && hh < h && ww >= 0 && ww < w)
+                code = get_code(x, ((img * h + hh) * w + ww) * c + cc, bits, is_signed);
+        }
+        y[e] = static_cast<uint8_t>(code & 0xFF);
+    }
+}
+
+// chsum[pix] = sum_c (x[pix, c] - zx) over the true channels of every input pixel.
+__global__ void __launch_bounds__(256) chsum_kernel(const uint8_t *__restrict__ x, int32_t *__restrict__ chsum,
+                                                    int64_t npix, int32_t c, int32_t bits, int32_t is_signed,
+                                                    int32_t zx) {
+    const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    const int64_t nwarps = (static_cast<int64_t>(gridDim.x) * blockDim.x) >> 5;
+    for (int64_t pix = warp; pix < npix; pix += nwarps) {
+        int32_t s = 0;
+        for (int32_t ch = lane; ch < c; ch += 32) s += get_code(x, pix * c + ch, bits, is_signed) - zx;
+        for (int off = 16; off > 0; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
+        if (lane == 0) chsum[pix] = s;
+    }
+}
+
+// x1[m] = sum over the in-bounds taps (r, s) of output pixel m of chsum[input pixel]:
+// sum_{taps, c} (x - zx) with padded taps contributing nothing (Z2).
+__global__ void __launch_bounds__(256) x1_kernel(const int32_t *__restrict__ chsum, int32_t *__restrict__ x1,
+                                                 int32_t n, int32_t h, int32_t w, int32_t P, int32_t Q,
+                                                 int32_t R, int32_t S, int32_t sh, int32_t sw, int32_t ph,
+                                                 int32_t pw, int32_t dh, int32_t dw) {
+    const int64_t M = static_cast<int64_t>(n) * P * Q;
+    for (int64_t m = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; m < M;
+         m += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t img = m / (static_cast<int64_t>(P) * Q);
+        const int32_t rem = static_cast<int32_t>(m - img * P * Q);
+        const int32_t p = rem / Q, q = rem - (rem / Q) * Q;
+        int32_t s = 0;
+        for (int32_t r = 0; r < R; ++r) {
+            const int32_t hh = p * sh - ph + r * dh;
+            if (hh < 0 || hh >= h) continue;
+            for (int32_t t = 0; t < S; ++t) {
+                const int32_t ww = q * sw - pw + t * dw;
+                if (ww < 0 || ww >= w) continue;
+                s += chsum[(img * h + hh) * w + ww];
             }
         }
-        __syncthreads();
-        for (int32_t j = threadIdx.x; j < p.ws; j += blockDim.x) {
-            uint32_t wv[4] = {0u, 0u, 0u, 0u};
-#pragma unroll
-            for (int jj = 0; jj < 16; ++jj) {
-                int32_t code = p.z;
-                if (jj < 4 * p.c) {
-                    const int32_t blkc = jj / p.c, cc = jj - blkc * p.c;
-                    const int32_t hh = 2 * i + (blkc >> 1) - p.pad_h;
-                    const int32_t ww = 2 * j + (blkc & 1) - p.pad_w;
-                    if (hh >= 0 && hh < p.h && ww >= 0 && ww < p.w)
-                        code = quantize_one(rows[blkc >> 1][ww * p.c + cc], qp);
-                }
-                wv[jj >> 2] |= static_cast<uint32_t>(code & 0xFF) << (8 * (jj & 3));
-            }
-            *reinterpret_cast<uint4 *>(p.y + ((img * p.hs + i) * p.ws + j) * 16) =
-                make_uint4(wv[0], wv[1], wv[2], wv[3]);
-        }
+        x1[m] = s;
     }
 }
 
@@ -334,6 +435,27 @@ __global__ void __launch_bounds__(256) weights_s2d_kernel(const uint8_t *__restr
         }
         w2[e] = static_cast<int8_t>(v);
     }
+}
+
+// Debug: one im2col TMA tile straight to global memory (no swizzle).
+__global__ void qconv_debug_im2col_kernel(const __grid_constant__ CUtensorMap xmap, int32_t c,
+                                          int32_t w, int32_t h, int32_t n, uint16_t ow,
+                                          uint16_t oh, uint32_t bytes, uint8_t *out) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                                ~uintptr_t(1023));
+    __shared__ __align__(8) uint64_t bar;
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        mbar_arrive_expect_tx(&bar, bytes);
+        tma_load_im2col_4d(smem, &xmap, &bar, c, w, h, n, ow, oh);
+    }
+    mbar_wait(&bar, 0);
+    for (uint32_t i = threadIdx.x; i < bytes; i += blockDim.x) out[i] = smem[i];
 }
 
 }  // namespace qc

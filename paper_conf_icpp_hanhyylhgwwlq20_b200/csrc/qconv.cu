@@ -1,27 +1,29 @@
 // qconv.cu -- host side of libqconv.so: the C ABI declared in include/qconv.h.
 //
-// Validation, the overflow bound, the per-shape launch plan (tile sizes,
-// pipeline depth, shared-memory carve-up), TMA descriptor encoding (im2col
-// for activations, tiled for weights) and kernel launches.  All device work
-// is in conv_fwd.cuh / prep.cuh.  Nothing here allocates device memory.
+// Validation, the overflow bound, the rewrite of a descriptor into the form the kernels
+// take ("exec" descriptor: channel padding / space-to-depth for channel counts the kernels
+// cannot take directly), the per-shape launch plan (kernel family, tile sizes, pipeline
+// depth, shared-memory carve-up) with the tuning hooks of the paper's profile-run search
+// (P:L271-273), TMA descriptor encoding and kernel launches (launch.h, k_*.cu).  All device
+// work is in conv_fwd.cuh / halo.cuh / trans.cuh / fwd2.cuh / prep.cuh.  Nothing here
+// allocates device memory.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cmath>
 #include <cstdint>
-#include <cstring>
-#include <mutex>
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <string>
 #include <vector>
 
 #include "qconv.h"
-#include "conv_fwd.cuh"
+#include "launch.h"
 #include "prep.cuh"
-#include "halo.cuh"
-#include "trans.cuh"
-#include "fwd2.cuh"
 
 namespace {
 
@@ -33,9 +35,17 @@ qc_status cuda_fail(cudaError_t e) {
 }
 
 bool is_int_input(qc_dtype t) { return t == QC_U4 || t == QC_S4 || t == QC_U8 || t == QC_S8; }
-bool is_valid_dtype(qc_dtype t) { return is_int_input(t) || t == QC_S32; }
-int dtype_bits(qc_dtype t) { return (t == QC_U4 || t == QC_S4) ? 4 : (t == QC_S32 ? 32 : 8); }
-bool dtype_signed(qc_dtype t) { return t == QC_S4 || t == QC_S8 || t == QC_S32; }
+bool is_float_out(qc_dtype t) { return t == QC_F32_OUT || t == QC_BF16_OUT; }
+bool is_packed_out(qc_dtype t) { return is_int_input(t); }
+int dtype_bits(qc_dtype t) {
+    switch (t) {
+        case QC_U4: case QC_S4: return 4;
+        case QC_U8: case QC_S8: return 8;
+        case QC_BF16_OUT: return 16;
+        default: return 32;
+    }
+}
+bool dtype_signed(qc_dtype t) { return t != QC_U4 && t != QC_U8; }
 int64_t dtype_min(qc_dtype t) {
     switch (t) {
         case QC_U4: return 0;
@@ -54,10 +64,22 @@ int64_t dtype_max(qc_dtype t) {
         default: return INT32_MAX;
     }
 }
+int out_kind(qc_dtype t) {
+    switch (t) {
+        case QC_U8: return qc::OUT_U8;
+        case QC_S8: return qc::OUT_S8;
+        case QC_U4: return qc::OUT_U4;
+        case QC_S4: return qc::OUT_S4;
+        case QC_F32_OUT: return qc::OUT_F32;
+        case QC_BF16_OUT: return qc::OUT_BF16;
+        default: return qc::OUT_S32;
+    }
+}
+qc_dtype byte_container(qc_dtype t) { return (t == QC_U4 || t == QC_U8) ? QC_U8 : QC_S8; }
 bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
 // MMA operand signedness of the activations: 4-bit codes are widened to unsigned bytes
-// (nibble-plane widening, conv_fwd.cuh widen_word); 8-bit codes are used as they are.
+// (nibble-plane widening, epilogue.cuh widen_word); 8-bit codes are used as they are.
 bool act_signed(const qconv_desc *d) { return dtype_bits(d->x_t) == 8 && dtype_signed(d->x_t); }
 
 // ------------------------------------------------------------------ driver entry points
@@ -98,9 +120,9 @@ const Driver &driver() {
     return d;
 }
 
-// Driver releases up to 13.1 mis-handle a descriptor flag for tensors under
-// 128 KiB; clearing bit 21 of the second descriptor word is the documented
-// workaround used by NVIDIA's own TMA helpers.
+// Driver releases up to 13.1 mis-handle a descriptor flag for tensors under 128 KiB;
+// clearing bit 21 of the second descriptor word is the workaround CUTLASS applies
+// (cute/atom/copy_traits_sm90_im2col.hpp, same version / size constants).
 void small_tensor_fixup(CUtensorMap *m, uint64_t tensor_bytes) {
     if (driver().driver_version <= 13010 && tensor_bytes < 131072)
         reinterpret_cast<uint64_t *>(m)[1] &= ~(1ull << 21);
@@ -123,34 +145,37 @@ int num_sms() {
 struct Geometry {
     int P, Q;
     int64_t M;
-    int bits;
+    int bits;           // activation bits
     int c_bytes;        // packed bytes per input pixel
     int64_t x_bytes, w_bytes, w8_bytes, y_bytes;
 };
 
-qc_status validate_desc(const qconv_desc *d, Geometry *g) {
+qc_status validate_desc(const qconv_desc *d, Geometry *g, bool allow_float) {
     if (!d) return QC_ERR_INVALID_ARG;
     if (d->n < 1 || d->h < 1 || d->w < 1 || d->c < 1 || d->k < 1 || d->r < 1 || d->s < 1)
         return QC_ERR_INVALID_ARG;
     if (d->stride_h < 1 || d->stride_w < 1 || d->dil_h < 1 || d->dil_w < 1 || d->pad_h < 0 ||
         d->pad_w < 0)
         return QC_ERR_INVALID_ARG;
-    if (!is_int_input(d->x_t) || !is_int_input(d->w_t) || !is_valid_dtype(d->y_t))
+    if (!is_int_input(d->x_t) || !is_int_input(d->w_t)) return QC_ERR_INVALID_ARG;
+    if (!(is_packed_out(d->y_t) || d->y_t == QC_S32 || (allow_float && is_float_out(d->y_t))))
         return QC_ERR_INVALID_ARG;
-    const int P = (d->h + 2 * d->pad_h - d->dil_h * (d->r - 1) - 1) / d->stride_h + 1;
-    const int Q = (d->w + 2 * d->pad_w - d->dil_w * (d->s - 1) - 1) / d->stride_w + 1;
-    if (d->h + 2 * d->pad_h - d->dil_h * (d->r - 1) - 1 < 0 ||
-        d->w + 2 * d->pad_w - d->dil_w * (d->s - 1) - 1 < 0 || P < 1 || Q < 1)
-        return QC_ERR_INVALID_ARG;
+    if (d->rounding != QC_ROUND_SINGLE && d->rounding != QC_ROUND_TFLITE) return QC_ERR_INVALID_ARG;
+    if (d->relu != 0 && d->relu != 1) return QC_ERR_INVALID_ARG;
+    const int64_t hx = static_cast<int64_t>(d->h) + 2 * d->pad_h - static_cast<int64_t>(d->dil_h) * (d->r - 1) - 1;
+    const int64_t wx = static_cast<int64_t>(d->w) + 2 * d->pad_w - static_cast<int64_t>(d->dil_w) * (d->s - 1) - 1;
+    if (hx < 0 || wx < 0) return QC_ERR_INVALID_ARG;
+    const int P = static_cast<int>(hx / d->stride_h + 1);
+    const int Q = static_cast<int>(wx / d->stride_w + 1);
     if (d->x_zero < dtype_min(d->x_t) || d->x_zero > dtype_max(d->x_t)) return QC_ERR_INVALID_ARG;
-    if (d->y_t != QC_S32) {
+    if (is_packed_out(d->y_t)) {
         if (d->y_zero < dtype_min(d->y_t) || d->y_zero > dtype_max(d->y_t)) return QC_ERR_INVALID_ARG;
         if (d->clamp_lo > d->clamp_hi || d->clamp_lo < dtype_min(d->y_t) ||
             d->clamp_hi > dtype_max(d->y_t))
             return QC_ERR_INVALID_ARG;
     }
     const int bits = dtype_bits(d->x_t);
-    if (bits == 4 && (d->c % 2)) return QC_ERR_INVALID_ARG;
+    if (bits == 4 && (d->c % 2)) return QC_ERR_INVALID_ARG;   // 4-bit pixel rows must be whole bytes
     const int64_t M = static_cast<int64_t>(d->n) * P * Q;
     g->P = P;
     g->Q = Q;
@@ -159,45 +184,202 @@ qc_status validate_desc(const qconv_desc *d, Geometry *g) {
     g->c_bytes = d->c * bits / 8;
     g->x_bytes = static_cast<int64_t>(d->n) * d->h * d->w * g->c_bytes;
     g->w8_bytes = static_cast<int64_t>(d->k) * d->r * d->s * d->c;
-    g->w_bytes = g->w8_bytes * dtype_bits(d->w_t) / 8;
+    g->w_bytes = (g->w8_bytes * dtype_bits(d->w_t) + 7) / 8;
     const int yb = dtype_bits(d->y_t);
     if (yb == 4 && (d->k % 2)) return QC_ERR_UNSUPPORTED;
     g->y_bytes = M * d->k * yb / 8;
     return QC_OK;
 }
 
-// Support + overflow checks for the GPU path (after validate_desc).
-qc_status check_supported(const qconv_desc *d, const Geometry &g) {
-    if (dtype_bits(d->x_t) != dtype_bits(d->w_t)) return QC_ERR_UNSUPPORTED;   // mixed widths: NEXT
-    const bool pair = dtype_bits(d->x_t) == 8 && d->c == 16;   // 2 taps per 32-byte K-stage
-    if (d->c % 32 && !pair) return QC_ERR_UNSUPPORTED;   // MMA K granularity / 16-byte TMA strides
-    if (d->stride_h > 8 || d->stride_w > 8) return QC_ERR_UNSUPPORTED;   // TMA traversal stride
-    const int lw = -d->pad_w, lh = -d->pad_h;
-    const int uw = d->pad_w - d->dil_w * (d->s - 1), uh = d->pad_h - d->dil_h * (d->r - 1);
-    if (lw < -128 || lh < -128 || uw < -128 || uh < -128 || uw > 127 || uh > 127)
-        return QC_ERR_UNSUPPORTED;                     // rank-4 im2col corner range
-    if (d->dil_w * (d->s - 1) > 255 || d->dil_h * (d->r - 1) > 255) return QC_ERR_UNSUPPORTED;
-    if (g.M > INT32_MAX - 256 || d->n > 65535) return QC_ERR_UNSUPPORTED;
-    if (static_cast<int64_t>(d->r) * d->s * d->c > INT32_MAX / 2) return QC_ERR_UNSUPPORTED;
-    // int32 accumulation bound ("overflow well addressed"): both the raw MMA sum and the
-    // zero-point-centred sum must stay inside int32 for any codes of these dtypes.
+// int32 accumulation bound ("overflow well addressed") on the caller's descriptor:
+// both the raw MMA sum and the zero-point-centred sum must stay inside int32 for any codes
+// of these dtypes.
+qc_status check_overflow(const qconv_desc *d) {
     const int64_t T = static_cast<int64_t>(d->r) * d->s * d->c;
     const int64_t wmax = std::max(-dtype_min(d->w_t), dtype_max(d->w_t));
+    const int64_t wctr = dtype_max(d->w_t) - dtype_min(d->w_t);      // |w - w_zero| with any zero point
     const int64_t xraw = std::max(-dtype_min(d->x_t), dtype_max(d->x_t));
     const int64_t xctr = std::max(d->x_zero - dtype_min(d->x_t), dtype_max(d->x_t) - d->x_zero);
     // 4-bit activations are widened to 16 x (x [+ 8]) (nibble-plane widening): the MMA sum
     // is 16 x larger and must stay below 2^30 (the epilogue adds 16 * bias inside int32)
-    const double lim = dtype_bits(d->x_t) == 4 ? 67108864.0 /* 2^30 / 16 */ : 2147483647.0;
-    const double xw = dtype_bits(d->x_t) == 4 ? 15.0 : static_cast<double>(std::max(xraw, xctr));
-    if (static_cast<double>(T) * xraw * wmax > lim || static_cast<double>(T) * xctr * wmax > lim ||
+    const bool nib = dtype_bits(d->x_t) == 4;
+    const double lim = nib ? 67108864.0 /* 2^30 / 16 */ : 2147483647.0;
+    const double xw = nib ? 15.0 : static_cast<double>(std::max(xraw, xctr));
+    const double wz = d->w_zero ? static_cast<double>(wctr) : static_cast<double>(wmax);
+    if (static_cast<double>(T) * xraw * wmax > lim || static_cast<double>(T) * xctr * wz > lim ||
         static_cast<double>(T) * xw * wmax > lim)
         return QC_ERR_OVERFLOW_RISK;
     return QC_OK;
 }
 
-// ------------------------------------------------------------------ launch plan
+// Structural limits of the kernels on the exec descriptor.
+qc_status check_structure(const qconv_desc *e, const Geometry &g) {
+    const bool pair = dtype_bits(e->x_t) == 8 && e->c == 16;   // 2 taps per 32-byte K-stage
+    if (e->c % 32 && !pair) return QC_ERR_UNSUPPORTED;
+    if (e->stride_h > 8 || e->stride_w > 8) return QC_ERR_UNSUPPORTED;   // TMA traversal stride
+    const int lw = -e->pad_w, lh = -e->pad_h;
+    const int uw = e->pad_w - e->dil_w * (e->s - 1), uh = e->pad_h - e->dil_h * (e->r - 1);
+    if (lw < -128 || lh < -128 || uw < -128 || uh < -128 || uw > 127 || uh > 127)
+        return QC_ERR_UNSUPPORTED;                     // rank-4 im2col corner range
+    if (e->dil_w * (e->s - 1) > 255 || e->dil_h * (e->r - 1) > 255) return QC_ERR_UNSUPPORTED;
+    if (g.M > INT32_MAX - 256 || e->n > 65535) return QC_ERR_UNSUPPORTED;
+    if (static_cast<int64_t>(e->r) * e->s * e->c > INT32_MAX / 2) return QC_ERR_UNSUPPORTED;
+    return QC_OK;
+}
+
+// ------------------------------------------------------------------ exec descriptor
+enum Xform { XF_NONE = 0, XF_S2D = 1, XF_PAD = 2 };
+enum WPrep { WP_COPY = 0, WP_NIBBLE = 1, WP_PLAIN = 2, WP_S2D = 3 };
+
+struct Exec {
+    const qconv_desc *d;  // the caller's descriptor
+    Geometry gu;          // its geometry
+    qconv_desc e;         // what the conv kernel sees
+    Geometry g;           // its geometry
+    int xform;
+    int wprep;            // layout of the prepared weights
+    bool wprep_needed;    // unprepared weights that need preparation on this call
+    size_t prep_bytes;
+    bool zx, zw;
+    size_t off_w, off_x, off_zx, off_cs, off_x1, ws_total;
+    int prologue;         // qconv_plan.prologue mask
+};
+
+int32_t s2d_channels(int32_t c) {
+    const int32_t c4 = 4 * c;
+    return c4 <= 16 ? 16 : (c4 + 31) / 32 * 32;
+}
+
+// Space-to-depth descriptor of a stride-2 conv (qconv.h): stride-1, unpadded, ceil(r/2) x
+// ceil(s/2) taps over s2d_channels(c) byte codes; same output geometry.
+qconv_desc s2d_of(const qconv_desc *d, const Geometry &g) {
+    qconv_desc o = *d;
+    o.r = (d->r + 1) / 2;
+    o.s = (d->s + 1) / 2;
+    o.h = g.P + o.r - 1;
+    o.w = g.Q + o.s - 1;
+    o.c = s2d_channels(d->c);
+    o.stride_h = o.stride_w = 1;
+    o.pad_h = o.pad_w = 0;
+    o.dil_h = o.dil_w = 1;
+    o.x_t = byte_container(d->x_t);
+    o.w_t = byte_container(d->w_t);
+    o.w_prepared = 1;
+    return o;
+}
+
+qc_status derive_exec(const qconv_desc *d, bool allow_float, Exec *ex) {
+    qc_status s = validate_desc(d, &ex->gu, allow_float);
+    if (s != QC_OK) return s;
+    const int xbits = dtype_bits(d->x_t), wbits = dtype_bits(d->w_t);
+    if (xbits == 4 && wbits == 8) return QC_ERR_UNSUPPORTED;   // nibble-plane weights need 4-bit w
+    s = check_overflow(d);
+    if (s != QC_OK) return s;
+    ex->d = d;
+    ex->e = *d;
+    const bool direct = (d->c % 32 == 0) || (xbits == 8 && d->c == 16);
+    if (direct) {
+        ex->xform = XF_NONE;
+    } else if (d->stride_h == 2 && d->stride_w == 2 && d->dil_h == 1 && d->dil_w == 1 && 4 * d->c <= 16 &&
+               d->w_zero == nullptr) {
+        // (with weight zero points the s2d zero weights beyond r, s would not contribute 0)
+        ex->xform = XF_S2D;
+        ex->e = s2d_of(d, ex->gu);
+    } else {
+        ex->xform = XF_PAD;
+        ex->e.c = (xbits == 8 && d->c < 16) ? 16 : (d->c + 31) / 32 * 32;
+    }
+    qconv_desc &e = ex->e;
+    if (ex->xform == XF_S2D) ex->wprep = WP_S2D;
+    else if (xbits == 4) ex->wprep = WP_NIBBLE;
+    else if (wbits == 4 || ex->xform == XF_PAD) ex->wprep = WP_PLAIN;
+    else ex->wprep = WP_COPY;
+    if (ex->wprep == WP_PLAIN) e.w_t = byte_container(d->w_t);
+    s = validate_desc(&e, &ex->g, allow_float);
+    if (s != QC_OK) return s;
+    s = check_structure(&e, ex->g);
+    if (s != QC_OK) return s;
+    const size_t w8 = static_cast<size_t>(ex->g.w8_bytes);
+    ex->prep_bytes = ex->wprep == WP_NIBBLE ? align_up(w8, 16) + 4 * static_cast<size_t>(e.k) : w8;
+    ex->wprep_needed = !d->w_prepared && ex->wprep != WP_COPY;
+    ex->zx = e.x_zero != 0;
+    ex->zw = d->w_zero != nullptr;
+    size_t off = 0;
+    ex->off_w = ex->off_x = ex->off_zx = ex->off_cs = ex->off_x1 = 0;
+    ex->prologue = 0;
+    if (ex->wprep_needed) { ex->off_w = off; off += align_up(ex->prep_bytes, 256); ex->prologue |= 1; }
+    if (ex->xform != XF_NONE) { ex->off_x = off; off += align_up(static_cast<size_t>(ex->g.x_bytes), 256); ex->prologue |= 2; }
+    if (ex->zx) {
+        ex->off_zx = off;
+        off += align_up(static_cast<size_t>(e.k) * (e.r + 1) * (e.s + 1) * 4, 256);
+        ex->prologue |= 4;
+    }
+    if (ex->zw) {
+        ex->off_cs = off;
+        off += align_up(static_cast<size_t>(e.n) * e.h * e.w * 4, 256);
+        ex->off_x1 = off;
+        off += align_up(static_cast<size_t>(ex->g.M) * 4, 256);
+        ex->prologue |= 8;
+    }
+    ex->ws_total = off;
+    return QC_OK;
+}
+
+// Weight preparation into the exec layout (qconv_prepare_weights and the prologue).
+qc_status prepare_weights_exec(const Exec &ex, const void *w, void *out, cudaStream_t st) {
+    const qconv_desc *d = ex.d;
+    const qconv_desc &e = ex.e;
+    const int64_t rows = static_cast<int64_t>(d->k) * d->r * d->s;
+    const int sgn = dtype_signed(d->w_t) ? 1 : 0;
+    switch (ex.wprep) {
+        case WP_COPY: {
+            cudaError_t err = cudaMemcpyAsync(out, w, static_cast<size_t>(ex.g.w8_bytes), cudaMemcpyDeviceToDevice, st);
+            if (err != cudaSuccess) return cuda_fail(err);
+            break;
+        }
+        case WP_NIBBLE: {
+            if (e.c == d->c) {
+                const int64_t ngroups = ex.gu.w_bytes / 16;
+                const int grid = static_cast<int>(std::min<int64_t>((ngroups + 255) / 256, 4096));
+                qc::widen_w4_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(w), static_cast<int8_t *>(out),
+                                                          ngroups, sgn);
+            } else {
+                const int64_t ngroups = rows * (e.c / 32);
+                const int grid = static_cast<int>(std::min<int64_t>((ngroups + 255) / 256, 4096));
+                qc::widen_w4_pad_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(w),
+                                                              static_cast<int8_t *>(out), rows, d->c, e.c, sgn);
+            }
+            int32_t *wsum = reinterpret_cast<int32_t *>(static_cast<uint8_t *>(out) +
+                                                        align_up(static_cast<size_t>(ex.g.w8_bytes), 16));
+            qc::wsum_w4_kernel<<<d->k, 256, 0, st>>>(static_cast<const uint8_t *>(w), wsum,
+                                                     static_cast<int64_t>(d->r) * d->s * d->c / 2, sgn);
+            break;
+        }
+        case WP_PLAIN: {
+            const int64_t total = rows * e.c;
+            const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, 4096));
+            qc::weights_plain_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(w), static_cast<int8_t *>(out),
+                                                           rows, d->c, e.c, dtype_bits(d->w_t), sgn);
+            break;
+        }
+        case WP_S2D: {
+            const int64_t total = static_cast<int64_t>(e.k) * e.r * e.s * e.c;
+            const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, 4096));
+            qc::weights_s2d_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(w), static_cast<int8_t *>(out),
+                                                         d->k, d->r, d->s, d->c, e.r, e.s, e.c,
+                                                         dtype_bits(d->w_t), sgn);
+            break;
+        }
+    }
+    cudaError_t err = cudaGetLastError();
+    if (err != cudaSuccess) return cuda_fail(err);
+    return QC_OK;
+}
+
+// ------------------------------------------------------------------ launch plans
 struct Plan {
-    int BK, bkp, chunks, BN, n_tiles_n, num_tiles, num_kb, stages, grid, threads;
+    int kernel;       // qc_kernel
+    int BK, bkp, chunks, BN, BM, n_tiles_n, num_tiles, num_kb, stages, grid, threads;
     uint32_t tmem_cols, smem_bytes;
     qc::ConvParams cp;
 };
@@ -208,23 +390,34 @@ uint32_t pow2_cols(int n) {
     while (c < static_cast<uint32_t>(n)) c <<= 1;
     return c;
 }
+bool needs_general_only(const Exec &ex) {
+    return ex.zx || ex.zw || !is_packed_out(ex.e.y_t);
+}
 
-qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
+// im2col kernel (conv_fwd.cuh).  bn_req = 0: the default N tile (largest <= 256, halved
+// while the grid would not fill the GPU -- P:L321: at small batch the tiling decides how
+// well the machine is filled).
+bool make_plan(const qconv_desc *d, const Geometry &g, int bn_req, Plan *pl) {
     const bool is4 = g.bits == 4;
     const bool pair = !is4 && d->c == 16;
+    pl->kernel = QC_KERNEL_IM2COL;
     pl->BK = pair ? 32 : choose_bk(d->c);
     pl->bkp = is4 ? pl->BK / 2 : (pair ? 16 : pl->BK);
     pl->chunks = pair ? 1 : d->c / pl->BK;
     pl->num_kb = pair ? (d->r * d->s + 1) / 2 : d->r * d->s * pl->chunks;
     const int m_tiles = static_cast<int>((g.M + qc::kBM - 1) / qc::kBM);
     const int sms = num_sms();
-    int BN = std::min(qc::kMaxBN, ((d->k + 15) / 16) * 16);
-    // smaller N tiles when the grid would not fill the GPU (paper P:L321: at small batch the
-    // tiling decides how well the machine is filled)
-    while (BN > 64 && static_cast<int64_t>(m_tiles) * ((d->k + BN - 1) / BN) < sms) {
-        BN = std::max(64, ((BN / 2 + 15) / 16) * 16);
+    int BN;
+    if (bn_req > 0) {
+        if (bn_req % 16 || bn_req > qc::kMaxBN) return false;
+        BN = bn_req;
+    } else {
+        BN = std::min(qc::kMaxBN, ((d->k + 15) / 16) * 16);
+        while (BN > 64 && static_cast<int64_t>(m_tiles) * ((d->k + BN - 1) / BN) < sms)
+            BN = std::max(64, ((BN / 2 + 15) / 16) * 16);
     }
     pl->BN = BN;
+    pl->BM = qc::kBM;
     pl->n_tiles_n = (d->k + BN - 1) / BN;
     pl->num_tiles = m_tiles * pl->n_tiles_n;
     pl->tmem_cols = pow2_cols(2 * BN);
@@ -232,11 +425,11 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const uint32_t b_bytes = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * pl->BK, 1024));
     const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(qc::kBM * pl->bkp) : 0u;
     const uint32_t per_stage = a_bytes + b_bytes + stg_bytes;
+    const bool packed = is_packed_out(d->y_t);
     const int ybits = dtype_bits(d->y_t);
     const int tile_row_bytes = BN * ybits / 8;
     const int y_gw = tile_row_bytes >= 128 ? 128 : tile_row_bytes;
-    const bool y_tma = d->y_t != QC_S32 && BN % 32 == 0 &&
-                       (static_cast<int64_t>(d->k) * ybits / 8) % 16 == 0 &&
+    const bool y_tma = packed && BN % 32 == 0 && (static_cast<int64_t>(d->k) * ybits / 8) % 16 == 0 &&
                        (y_gw == 32 || y_gw == 64 || (y_gw == 128 && tile_row_bytes % 128 == 0));
     const uint32_t ystg_one = y_tma ? 128u * static_cast<uint32_t>(tile_row_bytes) : 0u;
     const uint32_t ystg_bytes = 2u * ystg_one;   // double-buffered
@@ -244,7 +437,7 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const uint32_t budget = 227u * 1024u - 1024u - fixed;
     int stages = static_cast<int>(budget / per_stage);
     stages = std::min(stages, 32);     // deep rings: TMA latency is ~1-3 us under load
-    if (stages < 2) return QC_ERR_UNSUPPORTED;
+    if (stages < 2) return false;
     pl->stages = stages;
     qc::ConvParams &p = pl->cp;
     std::memset(&p, 0, sizeof(p));
@@ -293,16 +486,16 @@ qc_status make_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.sw_layout = pl->BK == 128 ? 2 : (pl->BK == 64 ? 4 : 6);
     p.pair = pair ? 1 : 0;
     p.cvt_shift = pl->bkp >= 64 ? 2 : (pl->bkp >= 32 ? 1 : 0);
-    p.need_clamp = (d->y_t != QC_S32 && (d->clamp_lo > dtype_min(d->y_t) || d->clamp_hi < dtype_max(d->y_t))) ? 1 : 0;
+    p.need_clamp = (packed && (d->clamp_lo > dtype_min(d->y_t) || d->clamp_hi < dtype_max(d->y_t))) ? 1 : 0;
     p.sw_mask = pl->BK == 128 ? 7 : (pl->BK == 64 ? 3 : 1);
     p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), act_signed(d), dtype_signed(d->w_t));
     p.tmem_cols = pl->tmem_cols;
-    p.y_zero = d->y_t == QC_S32 ? 0 : d->y_zero;
-    p.clamp_lo = d->y_t == QC_S32 ? INT32_MIN : d->clamp_lo;
-    p.clamp_hi = d->y_t == QC_S32 ? INT32_MAX : d->clamp_hi;
+    p.y_zero = packed ? d->y_zero : 0;
+    p.clamp_lo = packed ? d->clamp_lo : INT32_MIN;
+    p.clamp_hi = packed ? d->clamp_hi : INT32_MAX;
     p.x_zero = d->x_zero;
     p.y_row_bytes = static_cast<int64_t>(d->k) * dtype_bits(d->y_t) / 8;
-    return QC_OK;
+    return true;
 }
 
 CUtensorMapSwizzle swizzle_for(int bk) {
@@ -396,93 +589,19 @@ qc_status encode_y_map(const qconv_desc *d, const Geometry &g, void *y, int gw, 
     return QC_OK;
 }
 
-// Programmatic dependent launch (see ptx.cuh griddep_wait): the conv kernels may start while
-// the previous kernel of the stream drains; QC_NO_PDL=1 disables it (debug).
-void set_pdl(cudaLaunchConfig_t &cfg, cudaLaunchAttribute *attr) {
-    static const bool off = std::getenv("QC_NO_PDL") != nullptr;
-    if (off) return;
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-}
-
-// Debug hooks (never set in normal use): QC_EXPERIMENT=<flags> ablations, and
-// QC_TRACE=<file> timestamps of CTA 0's pipeline events, appended to the file after a sync.
-qc::ConvParams debug_params(const qc::ConvParams &base, cudaStream_t stream) {
-    static const char *trace_file = std::getenv("QC_TRACE");
-    static const char *exp_env = std::getenv("QC_EXPERIMENT");
-    qc::ConvParams cp = base;
-    cp.exp_flags = exp_env ? std::atoi(exp_env) : 0;
-    cp.trace = nullptr;
-    if (trace_file) {
-        unsigned long long *tbuf = nullptr;
-        cudaMalloc(&tbuf, 16 * 1024 * sizeof(unsigned long long));
-        cudaMemsetAsync(tbuf, 0, 16 * 1024 * sizeof(unsigned long long), stream);
-        cp.trace = tbuf;
-    }
-    return cp;
-}
-
-void debug_dump(const qc::ConvParams &cp, cudaStream_t stream) {
-    if (!cp.trace) return;
-    std::vector<unsigned long long> h(16 * 1024);
-    cudaMemcpyAsync(h.data(), cp.trace, h.size() * 8, cudaMemcpyDeviceToHost, stream);
-    cudaStreamSynchronize(stream);
-    cudaFree(cp.trace);
-    if (FILE *f = std::fopen(std::getenv("QC_TRACE"), "ab")) {
-        std::fwrite(h.data(), 8, h.size(), f);
-        std::fclose(f);
-    }
-}
-
-template <bool IS4, int OUT, bool ZX>
-qc_status launch_conv_t(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
-                        const CUtensorMap &ym, cudaStream_t stream) {
-    auto kern = qc::qconv_fwd_kernel<IS4, OUT, ZX>;
-    static int configured_smem = 0;   // per instantiation; max over calls is safe to keep
-    if (configured_smem < static_cast<int>(pl.smem_bytes)) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             227 * 1024);
-        if (e != cudaSuccess) return cuda_fail(e);
-        configured_smem = 227 * 1024;
-    }
-    cudaLaunchConfig_t cfg;
-    std::memset(&cfg, 0, sizeof(cfg));
-    cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
-    cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
-    cfg.dynamicSmemBytes = pl.smem_bytes;
-    cfg.stream = stream;
-    cudaLaunchAttribute pdl[1];
-    set_pdl(cfg, pdl);
-    qc::ConvParams cp = debug_params(pl.cp, stream);
-    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
-    if (e != cudaSuccess) return cuda_fail(e);
-    debug_dump(cp, stream);
-    return QC_OK;
-}
-
-template <bool IS4, int OUT>
-qc_status launch_conv(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
-                      const CUtensorMap &ym, cudaStream_t stream) {
-    return pl.cp.x_zero != 0 ? launch_conv_t<IS4, OUT, true>(pl, xm, wm, ym, stream)
-                             : launch_conv_t<IS4, OUT, false>(pl, xm, wm, ym, stream);
-}
-
-// ------------------------------------------------------------------ CTA-pair im2col (experimental)
-// The CTA-pair kernel (fwd2.cuh) runs im2col layers with R*S > 1 and a full N = 256 tile
-// (measured faster there: res4/res5 3x3 -6 to -13 % at 4 and 8 bits; no gain for 1x1 layers,
-// slower for N = 128 tiles).  QC_CTA2=1 forces it for every eligible layer (tests),
-// QC_NO_CTA2=1 disables it.
-bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, Plan *pl) {
-    static const bool force = std::getenv("QC_CTA2") != nullptr;
-    static const bool off = std::getenv("QC_NO_CTA2") != nullptr;
-    if (off) return false;
-    if (pl1.cp.pair || d->x_zero != 0 || d->y_t == QC_S32 || !pl1.cp.y_tma) return false;
+// ------------------------------------------------------------------ CTA-pair im2col
+// The CTA-pair kernel (fwd2.cuh) by default runs im2col layers with R*S > 1 and a full
+// N = 256 tile (measured faster there: res4/res5 3x3 -6 to -13 % at 4 and 8 bits; no gain
+// for 1x1 layers, slower for N = 128 tiles); any N tile of 64..256 (multiple of 32) can be
+// chosen through the plan API.
+bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, bool chosen, Plan *pl) {
+    if (pl1.cp.pair || d->x_zero != 0 || !is_packed_out(d->y_t) || !pl1.cp.y_tma) return false;
     const int BN = pl1.BN;
     if (BN % 32 || BN < 64) return false;
-    if (!force && !(BN == 256 && d->r * d->s > 1)) return false;
+    if (!chosen && !(BN == 256 && d->r * d->s > 1)) return false;
     *pl = pl1;
+    pl->kernel = QC_KERNEL_PAIR;
+    pl->BM = 2 * qc::kBM;
     qc::ConvParams &p = pl->cp;
     const bool is4 = g.bits == 4;
     const int m_tiles2 = static_cast<int>((g.M + 2 * qc::kBM - 1) / (2 * qc::kBM));
@@ -517,47 +636,10 @@ bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, Plan *p
     return true;
 }
 
-template <bool IS4, int OUT>
-qc_status launch_fwd2(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm, const CUtensorMap &ym,
-                      cudaStream_t stream) {
-    auto kern = qc::qconv_fwd2_kernel<IS4, OUT>;
-    static int configured = 0;
-    if (!configured) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        if (e != cudaSuccess) return cuda_fail(e);
-        configured = 1;
-    }
-    cudaLaunchConfig_t cfg;
-    std::memset(&cfg, 0, sizeof(cfg));
-    cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
-    cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
-    cfg.dynamicSmemBytes = pl.smem_bytes;
-    cfg.stream = stream;
-    cudaLaunchAttribute attr[2];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = 2;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    qc::ConvParams cp = debug_params(pl.cp, stream);
-    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
-    if (e != cudaSuccess) return cuda_fail(e);
-    debug_dump(cp, stream);
-    return QC_OK;
-}
-
 // ------------------------------------------------------------------ halo mode (stride 1)
-bool halo_disabled() {
-    static const bool off = std::getenv("QC_NO_HALO") != nullptr;
-    return off;
-}
-
-// Decide whether the stride-1 halo kernel applies and fill its plan.
 bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
-    if (halo_disabled()) return false;
     if (d->stride_h != 1 || d->stride_w != 1 || d->dil_h != 1 || d->dil_w != 1) return false;
-    if (d->x_zero != 0 || d->y_t == QC_S32) return false;
+    if (d->x_zero != 0 || !is_packed_out(d->y_t)) return false;
     const bool is4 = g.bits == 4;
     const int C8 = d->c;                                 // int8 bytes per pixel after widening
     const bool tap_pair = !is4 && C8 == 16;
@@ -579,7 +661,6 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const int KG8 = d->r * d->s * C8;
     const int nK = KG8 / 16;
     if (nK > 256) return false;
-    // N tile: largest of {round_up(K,32) <= 256, 128, 64, 32} whose weight slab fits in 100 KB
     // the whole weight slab stays resident (one N tile): MMA issue costs ~75 cycles per
     // instruction (measured), so narrower N tiles would be issue-bound
     if (d->k > 256) return false;
@@ -650,9 +731,11 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const int sms = num_sms();
     int grid = std::min<int64_t>(num_tiles, sms / n_tiles_n * n_tiles_n);
     grid = std::max(grid / n_tiles_n * n_tiles_n, n_tiles_n);
+    pl->kernel = QC_KERNEL_HALO;
     pl->grid = grid;
     pl->threads = is4 ? 512 : 384;
     pl->BN = BN;
+    pl->BM = qc::kBM;
     pl->n_tiles_n = n_tiles_n;
     pl->num_tiles = static_cast<int>(num_tiles);
     pl->stages = stages;
@@ -719,48 +802,24 @@ qc_status encode_halo_maps(const qconv_desc *d, const Geometry &g, const qc::Con
     return QC_OK;
 }
 
-template <bool IS4, int OUT>
-qc_status launch_halo(const Plan &pl, const CUtensorMap &hm, const CUtensorMap &bm,
-                      const CUtensorMap &ym, cudaStream_t stream) {
-    auto kern = qc::qconv_halo_kernel<IS4, OUT>;
-    static int configured = 0;
-    if (!configured) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        if (e != cudaSuccess) return cuda_fail(e);
-        configured = 1;
-    }
-    cudaLaunchConfig_t cfg;
-    std::memset(&cfg, 0, sizeof(cfg));
-    cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
-    cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
-    cfg.dynamicSmemBytes = pl.smem_bytes;
-    cfg.stream = stream;
-    cudaLaunchAttribute pdl[1];
-    set_pdl(cfg, pdl);
-    qc::ConvParams cp = debug_params(pl.cp, stream);
-    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, hm, bm, ym, cp);
-    if (e != cudaSuccess) return cuda_fail(e);
-    debug_dump(cp, stream);
-    return QC_OK;
-}
-
 // ------------------------------------------------------------------ channel-major 1x1 kernel
-bool trans_disabled() {
-    static const bool off = std::getenv("QC_NO_TRANS") != nullptr;
-    return off;
-}
-
-bool make_trans_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
-    if (trans_disabled()) return false;
-    if (d->r != 1 || d->s != 1 || d->x_zero != 0 || d->y_t == QC_S32) return false;
+// bmc_req = 0: 128 output channels per tile when k % 128 == 0, else 64.  With 4-bit
+// activations the 256-pixel operand tile doubles the on-chip widening per MAC; for deep
+// inputs (C > 512) that outweighs the cheaper epilogue (measured, r1), so the default
+// excludes them (the plan API can still choose it).
+bool make_trans_plan(const qconv_desc *d, const Geometry &g, int bmc_req, bool chosen, Plan *pl) {
+    if (d->r != 1 || d->s != 1 || d->x_zero != 0 || !is_packed_out(d->y_t)) return false;
     if (d->c % 32 || d->k % 64) return false;
     const bool is4 = g.bits == 4;
-    // With 4-bit activations the 256-pixel operand tile doubles the on-chip widening per
-    // MAC; for deep inputs (C > 512) that outweighs the cheaper epilogue (measured, r1).
-    if (is4 && d->c > 512) return false;
+    if (!chosen && is4 && d->c > 512) return false;
     const int ybits = dtype_bits(d->y_t);
     if ((static_cast<int64_t>(d->k) * ybits / 8) % 16) return false;
-    const int BMc = d->k % 128 == 0 ? 128 : 64;
+    int BMc = d->k % 128 == 0 ? 128 : 64;
+    if (bmc_req) {
+        if (bmc_req != 64 && bmc_req != 128) return false;
+        if (d->k % bmc_req) return false;
+        BMc = bmc_req;
+    }
     const int BNp = 256;
     const int BK = choose_bk(d->c);
     const int bkp = is4 ? BK / 2 : BK;
@@ -821,44 +880,310 @@ bool make_trans_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const int sms = num_sms();
     int grid = static_cast<int>(std::min<int64_t>(num_tiles, sms / n_tiles_n * n_tiles_n));
     grid = std::max(grid, 1);
+    pl->kernel = QC_KERNEL_CHANNEL;
     pl->grid = grid;
     pl->threads = is4 ? qc::kTThreads4 : qc::kTThreads8;
-    pl->BK = BK; pl->bkp = bkp; pl->BN = BMc; pl->n_tiles_n = n_tiles_n;
+    pl->BK = BK; pl->bkp = bkp; pl->BN = BMc; pl->BM = BNp; pl->n_tiles_n = n_tiles_n;
     pl->num_tiles = static_cast<int>(num_tiles); pl->stages = stages; pl->chunks = p.chunks;
     pl->num_kb = p.num_kb;
     return true;
 }
 
-template <bool IS4, int OUT, bool M64>
-qc_status launch_trans_m(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
-                         const CUtensorMap &ym, cudaStream_t stream) {
-    auto kern = qc::qconv_t_kernel<IS4, OUT, M64>;
-    static int configured = 0;
-    if (!configured) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-        if (e != cudaSuccess) return cuda_fail(e);
-        configured = 1;
+// ------------------------------------------------------------------ plan choice
+struct Choice {
+    int kernel = QC_KERNEL_AUTO;
+    int bn = 0;
+};
+
+// Resolve a choice to a plan on the exec descriptor; AUTO = the default rule
+// (halo -> channel-major -> CTA pair -> im2col).
+bool resolve(const Exec &ex, Choice c, Plan *pl) {
+    const qconv_desc *e = &ex.e;
+    const Geometry &g = ex.g;
+    const bool special_ok = !needs_general_only(ex);       // halo / channel / pair eligibility
+    if (c.kernel == QC_KERNEL_AUTO) {
+        if (special_ok && make_halo_plan(e, g, pl)) return true;
+        if (special_ok && make_trans_plan(e, g, 0, false, pl)) return true;
+        Plan p1;
+        if (!make_plan(e, g, 0, &p1)) return false;
+        if (special_ok && make_plan2(e, g, p1, false, pl)) return true;
+        *pl = p1;
+        return true;
     }
-    cudaLaunchConfig_t cfg;
-    std::memset(&cfg, 0, sizeof(cfg));
-    cfg.gridDim = dim3(static_cast<unsigned>(pl.grid));
-    cfg.blockDim = dim3(static_cast<unsigned>(pl.threads));
-    cfg.dynamicSmemBytes = pl.smem_bytes;
-    cfg.stream = stream;
-    cudaLaunchAttribute pdl[1];
-    set_pdl(cfg, pdl);
-    qc::ConvParams cp = debug_params(pl.cp, stream);
-    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, xm, wm, ym, cp);
-    if (e != cudaSuccess) return cuda_fail(e);
-    debug_dump(cp, stream);
+    switch (c.kernel) {
+        case QC_KERNEL_HALO:
+            if (!special_ok || !make_halo_plan(e, g, pl)) return false;
+            return c.bn == 0 || c.bn == pl->BN;
+        case QC_KERNEL_CHANNEL:
+            return special_ok && make_trans_plan(e, g, c.bn, true, pl);
+        case QC_KERNEL_PAIR: {
+            Plan p1;
+            return special_ok && make_plan(e, g, c.bn, &p1) && make_plan2(e, g, p1, true, pl);
+        }
+        case QC_KERNEL_IM2COL:
+            return make_plan(e, g, c.bn, pl);
+        default:
+            return false;
+    }
+}
+
+std::vector<Choice> candidates(const Exec &ex) {
+    std::vector<Choice> out;
+    Plan pl;
+    auto try_add = [&](int kernel, int bn) {
+        Choice c;
+        c.kernel = kernel;
+        c.bn = bn;
+        if (resolve(ex, c, &pl)) {
+            for (const Choice &o : out)
+                if (o.kernel == kernel && o.bn == pl.BN) return;
+            c.bn = pl.BN;
+            out.push_back(c);
+        }
+    };
+    try_add(QC_KERNEL_HALO, 0);
+    try_add(QC_KERNEL_CHANNEL, 64);
+    try_add(QC_KERNEL_CHANNEL, 128);
+    const int kmax = std::min(qc::kMaxBN, (ex.e.k + 15) / 16 * 16);
+    for (int bn : {64, 128, 256})
+        if (bn <= std::max(kmax, 64)) try_add(QC_KERNEL_PAIR, bn);
+    for (int bn : {32, 64, 128, 256})
+        if (bn < kmax * 2) try_add(QC_KERNEL_IM2COL, std::min(bn, kmax));
+    return out;
+}
+
+// Process-wide choices (qconv_plan_set) keyed by every field of the caller's descriptor
+// (w_zero by presence), and the autotuner's per-thread forced choice.
+std::mutex g_plan_mu;
+std::map<std::string, Choice> g_plans;
+thread_local bool g_forced = false;
+thread_local Choice g_force;
+
+std::string desc_key(const qconv_desc *d) {
+    const int32_t f[] = {d->n, d->h, d->w, d->c, d->k, d->r, d->s, d->stride_h, d->stride_w, d->pad_h,
+                         d->pad_w, d->dil_h, d->dil_w, static_cast<int32_t>(d->x_t), static_cast<int32_t>(d->w_t),
+                         static_cast<int32_t>(d->y_t), d->x_zero, d->w_zero ? 1 : 0, d->w_prepared, d->y_zero,
+                         d->clamp_lo, d->clamp_hi, d->rounding, d->relu};
+    return std::string(reinterpret_cast<const char *>(f), sizeof(f));
+}
+
+Choice current_choice(const qconv_desc *d) {
+    if (g_forced) return g_force;
+    std::lock_guard<std::mutex> lk(g_plan_mu);
+    if (g_plans.empty()) return Choice();
+    auto it = g_plans.find(desc_key(d));
+    return it == g_plans.end() ? Choice() : it->second;
+}
+
+void fill_plan_out(const Exec &ex, const Plan &pl, qconv_plan *o) {
+    std::memset(o, 0, sizeof(*o));
+    o->kernel = pl.kernel;
+    o->bn = pl.BN;
+    o->bm = pl.BM;
+    o->stages = pl.stages;
+    o->grid = pl.grid;
+    o->threads = pl.threads;
+    o->num_tiles = pl.num_tiles;
+    o->smem_bytes = static_cast<int32_t>(pl.smem_bytes);
+    o->tmem_cols = static_cast<int32_t>(pl.kernel == QC_KERNEL_HALO || pl.kernel == QC_KERNEL_CHANNEL
+                                            ? pl.cp.tmem_cols : pl.tmem_cols);
+    o->prologue = ex.prologue;
+    o->epilogue_mode = (needs_general_only(ex) || ex.e.rounding == QC_ROUND_TFLITE) ? 2 : -1;
+}
+
+// ------------------------------------------------------------------ the forward call
+qc_status run_prologue(const Exec &ex, const void *x, const void *w, void *ws, cudaStream_t st,
+                       const void **x_e, const void **w_e) {
+    const qconv_desc *d = ex.d;
+    const qconv_desc &e = ex.e;
+    uint8_t *wsb = static_cast<uint8_t *>(ws);
+    *x_e = x;
+    *w_e = w;
+    if (ex.wprep_needed) {
+        qc_status s = prepare_weights_exec(ex, w, wsb + ex.off_w, st);
+        if (s != QC_OK) return s;
+        *w_e = wsb + ex.off_w;
+    }
+    if (ex.xform == XF_S2D) {
+        const int64_t total = static_cast<int64_t>(e.n) * e.h * e.w * e.c;
+        const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, static_cast<int64_t>(num_sms()) * 16));
+        qc::repack_s2d_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(x), wsb + ex.off_x, d->n, d->h,
+                                                    d->w, d->c, e.h, e.w, e.c, d->pad_h, d->pad_w,
+                                                    dtype_bits(d->x_t), dtype_signed(d->x_t) ? 1 : 0, d->x_zero);
+        *x_e = wsb + ex.off_x;
+    } else if (ex.xform == XF_PAD) {
+        const int64_t npix = static_cast<int64_t>(d->n) * d->h * d->w;
+        const int64_t total = npix * ex.g.c_bytes;
+        const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, static_cast<int64_t>(num_sms()) * 16));
+        qc::repack_pad_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(x), wsb + ex.off_x, npix, d->c,
+                                                    e.c, dtype_bits(d->x_t), d->x_zero);
+        *x_e = wsb + ex.off_x;
+    }
+    if (ex.zx) {
+        int32_t *table = reinterpret_cast<int32_t *>(wsb + ex.off_zx);
+        qc::zx_table_kernel<<<(e.k + 127) / 128, 128, 0, st>>>(
+            static_cast<const int8_t *>(*w_e), table, e.k, e.r, e.s, e.c, dtype_signed(e.w_t) ? 0 : 1,
+            ex.wprep == WP_NIBBLE ? 1 : 0);
+    }
+    if (ex.zw) {
+        int32_t *cs = reinterpret_cast<int32_t *>(wsb + ex.off_cs);
+        int32_t *x1 = reinterpret_cast<int32_t *>(wsb + ex.off_x1);
+        const int64_t npix = static_cast<int64_t>(e.n) * e.h * e.w;
+        const int grid = static_cast<int>(std::min<int64_t>((npix * 32 + 255) / 256, static_cast<int64_t>(num_sms()) * 16));
+        qc::chsum_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(*x_e), cs, npix, e.c,
+                                               dtype_bits(e.x_t), dtype_signed(e.x_t) ? 1 : 0, e.x_zero);
+        const int grid2 = static_cast<int>(std::min<int64_t>((ex.g.M + 255) / 256, static_cast<int64_t>(num_sms()) * 16));
+        qc::x1_kernel<<<grid2, 256, 0, st>>>(cs, x1, e.n, e.h, e.w, ex.g.P, ex.g.Q, e.r, e.s, e.stride_h,
+                                             e.stride_w, e.pad_h, e.pad_w, e.dil_h, e.dil_w);
+    }
+    cudaError_t err = cudaGetLastError();
+    if (err != cudaSuccess) return cuda_fail(err);
     return QC_OK;
 }
 
-template <bool IS4, int OUT>
-qc_status launch_trans(const Plan &pl, const CUtensorMap &xm, const CUtensorMap &wm,
-                       const CUtensorMap &ym, cudaStream_t stream) {
-    return pl.BN == 64 ? launch_trans_m<IS4, OUT, true>(pl, xm, wm, ym, stream)
-                       : launch_trans_m<IS4, OUT, false>(pl, xm, wm, ym, stream);
+// Accumulator scale and signed-offset correction of 4-bit activations (widen_word).
+void set_act_params(const Exec &ex, const void *w8, qc::ConvParams &p) {
+    const bool nib = ex.wprep == WP_NIBBLE;
+    p.acc_lg = nib ? 4 : 0;
+    p.x_sgn4 = (nib && ex.e.x_t == QC_S4) ? 1 : 0;
+    p.wsum = p.x_sgn4 ? reinterpret_cast<const int32_t *>(static_cast<const uint8_t *>(w8) +
+                                                           align_up(static_cast<size_t>(ex.g.w8_bytes), 16))
+                      : nullptr;
+}
+
+#ifdef QC_DEBUG
+// Debug builds only: QC_TRACE=<file> appends timestamps of CTA 0's pipeline events after a sync.
+void debug_attach(qc::ConvParams &cp, cudaStream_t stream) {
+    static const char *trace_file = std::getenv("QC_TRACE");
+    cp.trace = nullptr;
+    if (trace_file) {
+        unsigned long long *tbuf = nullptr;
+        cudaMalloc(&tbuf, 16 * 1024 * sizeof(unsigned long long));
+        cudaMemsetAsync(tbuf, 0, 16 * 1024 * sizeof(unsigned long long), stream);
+        cp.trace = tbuf;
+    }
+}
+void debug_dump(const qc::ConvParams &cp, cudaStream_t stream) {
+    if (!cp.trace) return;
+    std::vector<unsigned long long> h(16 * 1024);
+    cudaMemcpyAsync(h.data(), cp.trace, h.size() * 8, cudaMemcpyDeviceToHost, stream);
+    cudaStreamSynchronize(stream);
+    cudaFree(cp.trace);
+    if (FILE *f = std::fopen(std::getenv("QC_TRACE"), "ab")) {
+        std::fwrite(h.data(), 8, h.size(), f);
+        std::fclose(f);
+    }
+}
+#else
+void debug_attach(qc::ConvParams &, cudaStream_t) {}
+void debug_dump(const qc::ConvParams &, cudaStream_t) {}
+#endif
+
+qc_status launch_plan(const Exec &ex, Plan &pl, const void *x, const void *w8, const int32_t *bias,
+                      const int32_t *mult, const int32_t *shift, const float *dq, void *y, void *ws,
+                      cudaStream_t st) {
+    const qconv_desc *e = &ex.e;
+    const Geometry &g = ex.g;
+    const bool is4 = g.bits == 4;
+    const int out = out_kind(e->y_t);
+    qc::ConvParams &p = pl.cp;
+    set_act_params(ex, w8, p);
+    p.bias = bias;
+    p.mult = mult;
+    p.shift = shift;
+    p.dq_scale = dq;
+    p.y = y;
+    p.round_tfl = e->rounding == QC_ROUND_TFLITE ? 1 : 0;
+    p.relu = e->relu;
+    uint8_t *wsb = static_cast<uint8_t *>(ws);
+    p.zx_table = ex.zx ? reinterpret_cast<const int32_t *>(wsb + ex.off_zx) : nullptr;
+    p.zw = ex.zw ? ex.d->w_zero : nullptr;
+    p.x1 = ex.zw ? reinterpret_cast<const int32_t *>(wsb + ex.off_x1) : nullptr;
+    debug_attach(p, st);
+    qc::Launch L;
+    L.grid = dim3(static_cast<unsigned>(pl.grid));
+    L.threads = pl.threads;
+    L.smem = pl.smem_bytes;
+    L.stream = st;
+    static const bool no_pdl = std::getenv("QC_NO_PDL") != nullptr;   // same bytes either way
+    L.pdl = !no_pdl;
+    cudaError_t err = cudaSuccess;
+    qc_status s = QC_OK;
+    alignas(64) CUtensorMap m0, m1, m2;
+    std::memset(&m2, 0, sizeof(m2));
+    switch (pl.kernel) {
+        case QC_KERNEL_HALO:
+            s = encode_halo_maps(e, g, p, x, w8, y, &m0, &m1, &m2);
+            if (s != QC_OK) return s;
+            err = qc::launch_halo(L, is4, out, m0, m1, m2, p);
+            break;
+        case QC_KERNEL_CHANNEL:
+            p.stg_sw = is4 ? packed_sw_mask(pl.bkp) : 0;
+            s = encode_x_map(e, g, x, pl.bkp, is4 ? packed_swizzle(pl.bkp) : swizzle_for(pl.BK), &m0, p.Wh);
+            if (s != QC_OK) return s;
+            s = encode_w_map_pairs(e, g, w8, pl.BK, pl.BN, swizzle_for(pl.BK), &m1);
+            if (s != QC_OK) return s;
+            s = encode_y_map(e, g, y, p.y_gw, &m2, p.Wh, true);
+            if (s != QC_OK) return s;
+            err = qc::launch_trans(L, is4, out, pl.BN == 64, m0, m1, m2, p);
+            break;
+        case QC_KERNEL_PAIR:
+        case QC_KERNEL_IM2COL: {
+            const bool pair = p.pair != 0;
+            p.stg_sw = is4 ? packed_sw_mask(pl.bkp) : 0;
+            s = encode_x_map(e, g, x, pl.bkp,
+                             pair ? CU_TENSOR_MAP_SWIZZLE_NONE : (is4 ? packed_swizzle(pl.bkp) : swizzle_for(pl.BK)),
+                             &m0);
+            if (s != QC_OK) return s;
+            const int wbn = pl.kernel == QC_KERNEL_PAIR ? pl.BN / 2 : pl.BN;
+            s = encode_w_map(e, g, w8, pair ? 16 : pl.BK, wbn, pair ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(pl.BK),
+                             &m1);
+            if (s != QC_OK) return s;
+            if (p.y_tma) {
+                s = encode_y_map(e, g, y, p.y_gw, &m2);
+                if (s != QC_OK) return s;
+            }
+            if (pl.kernel == QC_KERNEL_PAIR) {
+                L.cluster = 2;
+                err = qc::launch_fwd2(L, is4, out, m0, m1, m2, p);
+            } else {
+                err = qc::launch_fwd(L, is4, out, ex.zx || ex.zw, m0, m1, m2, p);
+            }
+            break;
+        }
+        default:
+            return QC_ERR_INVALID_ARG;
+    }
+    if (err != cudaSuccess) return cuda_fail(err);
+    debug_dump(p, st);
+    return QC_OK;
+}
+
+qc_status forward_impl(const qconv_desc *d, bool dequant, const void *x, const void *w, const int32_t *bias,
+                       const int32_t *mult, const int32_t *shift, const float *dq, void *y, void *workspace,
+                       size_t ws_bytes, void *stream) {
+    Exec ex;
+    qc_status s = derive_exec(d, dequant, &ex);
+    if (s != QC_OK) return s;
+    if (dequant && !is_float_out(d->y_t)) return QC_ERR_INVALID_ARG;
+    if (!x || !w || !y) return QC_ERR_INVALID_ARG;
+    if (is_packed_out(d->y_t) && (!mult || !shift)) return QC_ERR_INVALID_ARG;
+    if (dequant && !dq) return QC_ERR_INVALID_ARG;
+    if (!aligned16(x) || !aligned16(w) || !aligned16(y) || (bias && !aligned16(bias)) ||
+        (mult && !aligned16(mult)) || (shift && !aligned16(shift)) || (dq && !aligned16(dq)) ||
+        (d->w_zero && !aligned16(d->w_zero)) || (workspace && !aligned16(workspace)))
+        return QC_ERR_MISALIGNED;
+    if (ex.ws_total > 0 && (!workspace || ws_bytes < ex.ws_total)) return QC_ERR_WORKSPACE;
+    Plan pl;
+    const Choice c = current_choice(d);
+    if (!resolve(ex, c, &pl)) {
+        if (c.kernel == QC_KERNEL_AUTO || !resolve(ex, Choice(), &pl)) return QC_ERR_UNSUPPORTED;
+    }
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const void *x_e = nullptr, *w_e = nullptr;
+    s = run_prologue(ex, x, w, workspace, st, &x_e, &w_e);
+    if (s != QC_OK) return s;
+    return launch_plan(ex, pl, x_e, w_e, bias, mult, shift, dq, y, workspace, st);
 }
 
 }  // namespace
@@ -880,7 +1205,7 @@ const char *qconv_status_string(qc_status s) {
 }
 
 int qconv_last_cuda_error(void) { return g_last_cuda_error; }
-int qconv_version(void) { return 100; }
+int qconv_version(void) { return 200; }
 
 qc_status qconv_requant_params(float in_scale, const float *w_scale, float out_scale, int32_t k,
                                int32_t *multiplier, int32_t *shift) {
@@ -951,221 +1276,141 @@ qc_status qconv_quantize_pack(const void *x, qc_ftype xt, int64_t npix, int32_t 
     return QC_OK;
 }
 
-// Prepared weights: int8 KRSC (8-bit: the codes as they are; 4-bit: nibble-plane order,
-// prep.cuh widen_w4_kernel), then for 4-bit a 16-byte aligned int32 wsum[K].
-static size_t prepared_bytes(const qconv_desc *d, const Geometry &g) {
-    if (dtype_bits(d->w_t) == 8) return static_cast<size_t>(g.w8_bytes);
-    return align_up(static_cast<size_t>(g.w8_bytes), 16) + 4 * static_cast<size_t>(d->k);
-}
-static const int32_t *prepared_wsum(const qconv_desc *d, const Geometry &g, const void *w8) {
-    if (dtype_bits(d->w_t) != 4) return nullptr;
-    return reinterpret_cast<const int32_t *>(static_cast<const uint8_t *>(w8) +
-                                             align_up(static_cast<size_t>(g.w8_bytes), 16));
-}
-
 size_t qconv_prepared_weight_bytes(const qconv_desc *d) {
-    Geometry g;
-    if (validate_desc(d, &g) != QC_OK) return 0;
-    return prepared_bytes(d, g);
-}
-
-static qc_status prepare_weights_impl(const qconv_desc *d, const Geometry &g, const void *w,
-                                      void *w_prep, cudaStream_t st) {
-    if (dtype_bits(d->w_t) == 8) {
-        cudaError_t e = cudaMemcpyAsync(w_prep, w, static_cast<size_t>(g.w8_bytes),
-                                        cudaMemcpyDeviceToDevice, st);
-        if (e != cudaSuccess) return cuda_fail(e);
-        return QC_OK;
-    }
-    if (d->c % 32) return QC_ERR_UNSUPPORTED;            // nibble planes are 32-channel groups
-    const int64_t ngroups = g.w_bytes / 16;
-    const int grid = static_cast<int>(std::min<int64_t>((ngroups + 255) / 256, 4096));
-    const int sgn = d->w_t == QC_S4 ? 1 : 0;
-    qc::widen_w4_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(w),
-                                              static_cast<int8_t *>(w_prep), ngroups, sgn);
-    qc::wsum_w4_kernel<<<d->k, 256, 0, st>>>(
-        static_cast<const uint8_t *>(w), const_cast<int32_t *>(prepared_wsum(d, g, w_prep)),
-        static_cast<int64_t>(d->r) * d->s * d->c / 2, sgn);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return cuda_fail(e);
-    return QC_OK;
+    Exec ex;
+    if (derive_exec(d, true, &ex) != QC_OK) return 0;
+    return ex.prep_bytes;
 }
 
 qc_status qconv_prepare_weights(const qconv_desc *d, const void *w, void *w_prep, void *stream) {
-    Geometry g;
-    qc_status s = validate_desc(d, &g);
+    Exec ex;
+    qc_status s = derive_exec(d, true, &ex);
     if (s != QC_OK) return s;
     if (!w || !w_prep) return QC_ERR_INVALID_ARG;
     if (!aligned16(w) || !aligned16(w_prep)) return QC_ERR_MISALIGNED;
-    return prepare_weights_impl(d, g, w, w_prep, static_cast<cudaStream_t>(stream));
-}
-
-static size_t ws_weights_bytes(const qconv_desc *d, const Geometry &g) {
-    return (dtype_bits(d->w_t) == 4 && !d->w_prepared) ? align_up(prepared_bytes(d, g), 256) : 0;
-}
-static size_t ws_zx_bytes(const qconv_desc *d) {
-    return d->x_zero != 0 ? align_up(static_cast<size_t>(d->k) * (d->r + 1) * (d->s + 1) * 4, 256) : 0;
+    return prepare_weights_exec(ex, w, w_prep, static_cast<cudaStream_t>(stream));
 }
 
 size_t qconv2d_workspace_size(const qconv_desc *d) {
-    Geometry g;
-    if (validate_desc(d, &g) != QC_OK) return 0;
-    return ws_weights_bytes(d, g) + ws_zx_bytes(d);
-}
-
-// Accumulator scale and signed-offset correction of 4-bit activations (widen_word).
-static void set_act_params(const qconv_desc *d, const Geometry &g, const void *w8, qc::ConvParams &p) {
-    p.acc_lg = g.bits == 4 ? 4 : 0;
-    p.x_sgn4 = (g.bits == 4 && d->x_t == QC_S4) ? 1 : 0;
-    p.wsum = p.x_sgn4 ? prepared_wsum(d, g, w8) : nullptr;
+    Exec ex;
+    if (derive_exec(d, true, &ex) != QC_OK) return 0;
+    return ex.ws_total;
 }
 
 qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, const int32_t *bias,
                           const int32_t *multiplier, const int32_t *shift, void *y, void *workspace,
                           size_t ws_bytes, void *stream) {
-    Geometry g;
-    qc_status s = validate_desc(d, &g);
-    if (s != QC_OK) return s;
-    if (!x || !w || !y) return QC_ERR_INVALID_ARG;
-    if (d->y_t != QC_S32 && (!multiplier || !shift)) return QC_ERR_INVALID_ARG;
-    s = check_supported(d, g);
-    if (s != QC_OK) return s;
-    if (!aligned16(x) || !aligned16(w) || !aligned16(y) || (bias && !aligned16(bias)) ||
-        (multiplier && !aligned16(multiplier)) || (shift && !aligned16(shift)) ||
-        (workspace && !aligned16(workspace)))
-        return QC_ERR_MISALIGNED;
-    const size_t need_w = ws_weights_bytes(d, g), need_z = ws_zx_bytes(d);
-    if (need_w + need_z > 0 && (!workspace || ws_bytes < need_w + need_z)) return QC_ERR_WORKSPACE;
-    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    return forward_impl(d, false, x, w, bias, multiplier, shift, nullptr, y, workspace, ws_bytes, stream);
+}
 
+qc_status qconv2d_forward_dequant(const qconv_desc *d, const void *x, const void *w, const int32_t *bias,
+                                  const float *scale, void *y, void *workspace, size_t ws_bytes, void *stream) {
+    return forward_impl(d, true, x, w, bias, nullptr, nullptr, scale, y, workspace, ws_bytes, stream);
+}
+
+qc_status qconv_debug_plan(const qconv_desc *d, qconv_plan *out) {
+    if (!out) return QC_ERR_INVALID_ARG;
+    Exec ex;
+    qc_status s = derive_exec(d, true, &ex);
+    if (s != QC_OK) return s;
     Plan pl;
-    s = make_plan(d, g, &pl);
-    if (s != QC_OK) return s;
+    const Choice c = current_choice(d);
+    if (!resolve(ex, c, &pl)) {
+        if (c.kernel == QC_KERNEL_AUTO || !resolve(ex, Choice(), &pl)) return QC_ERR_UNSUPPORTED;
+    }
+    fill_plan_out(ex, pl, out);
+    return QC_OK;
+}
 
-    const void *w8 = w;
-    if (need_w) {
-        s = prepare_weights_impl(d, g, w, workspace, st);
-        if (s != QC_OK) return s;
-        w8 = workspace;
-    }
-    {   // stride-1 convolutions: halo kernel (one tiled TMA per tile, resident weights)
-        Plan hp;
-        if (need_z == 0 && make_halo_plan(d, g, &hp)) {
-            set_act_params(d, g, w8, hp.cp);
-            hp.cp.w_early = need_w == 0 ? 1 : 0;
-            hp.cp.bias = bias;
-            hp.cp.mult = multiplier;
-            hp.cp.shift = shift;
-            hp.cp.y = y;
-            alignas(64) CUtensorMap hm, bm, ym;
-            s = encode_halo_maps(d, g, hp.cp, x, w8, y, &hm, &bm, &ym);
-            if (s != QC_OK) return s;
-            const bool is4 = g.bits == 4;
-            switch (d->y_t) {
-                case QC_U8: return is4 ? launch_halo<true, qc::OUT_U8>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_U8>(hp, hm, bm, ym, st);
-                case QC_S8: return is4 ? launch_halo<true, qc::OUT_S8>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_S8>(hp, hm, bm, ym, st);
-                case QC_U4: return is4 ? launch_halo<true, qc::OUT_U4>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_U4>(hp, hm, bm, ym, st);
-                case QC_S4: return is4 ? launch_halo<true, qc::OUT_S4>(hp, hm, bm, ym, st) : launch_halo<false, qc::OUT_S4>(hp, hm, bm, ym, st);
-                default: break;
-            }
-        }
-    }
-    {   // 1x1 convolutions: channel-major kernel (per-channel constants in registers)
-        Plan tp;
-        if (need_z == 0 && make_trans_plan(d, g, &tp)) {
-            set_act_params(d, g, w8, tp.cp);
-            tp.cp.bias = bias;
-            tp.cp.mult = multiplier;
-            tp.cp.shift = shift;
-            tp.cp.y = y;
-            alignas(64) CUtensorMap xm, wm, ym;
-            tp.cp.stg_sw = g.bits == 4 ? packed_sw_mask(tp.bkp) : 0;
-            s = encode_x_map(d, g, x, tp.bkp, g.bits == 4 ? packed_swizzle(tp.bkp) : swizzle_for(tp.BK), &xm,
-                             tp.cp.Wh);
-            if (s != QC_OK) return s;
-            s = encode_w_map_pairs(d, g, w8, tp.BK, tp.BN, swizzle_for(tp.BK), &wm);
-            if (s != QC_OK) return s;
-            s = encode_y_map(d, g, y, tp.cp.y_gw, &ym, tp.cp.Wh, true);
-            if (s != QC_OK) return s;
-            const bool is4 = g.bits == 4;
-            switch (d->y_t) {
-                case QC_U8: return is4 ? launch_trans<true, qc::OUT_U8>(tp, xm, wm, ym, st) : launch_trans<false, qc::OUT_U8>(tp, xm, wm, ym, st);
-                case QC_S8: return is4 ? launch_trans<true, qc::OUT_S8>(tp, xm, wm, ym, st) : launch_trans<false, qc::OUT_S8>(tp, xm, wm, ym, st);
-                case QC_U4: return is4 ? launch_trans<true, qc::OUT_U4>(tp, xm, wm, ym, st) : launch_trans<false, qc::OUT_U4>(tp, xm, wm, ym, st);
-                case QC_S4: return is4 ? launch_trans<true, qc::OUT_S4>(tp, xm, wm, ym, st) : launch_trans<false, qc::OUT_S4>(tp, xm, wm, ym, st);
-                default: break;
-            }
-        }
-    }
-    qc::ConvParams &p = pl.cp;
-    set_act_params(d, g, w8, p);
-    if (need_z) {
-        int32_t *table = reinterpret_cast<int32_t *>(static_cast<uint8_t *>(workspace) + need_w);
-        qc::zx_table_kernel<<<(d->k + 127) / 128, 128, 0, st>>>(
-            static_cast<const int8_t *>(w8), table, d->k, d->r, d->s, d->c, dtype_signed(d->w_t) ? 0 : 1,
-            g.bits == 4 ? 1 : 0);
-        cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess) return cuda_fail(e);
-        p.zx_table = table;
-    }
-    p.bias = bias;
-    p.mult = multiplier;
-    p.shift = shift;
-    p.y = y;
-
-    alignas(64) CUtensorMap xm, wm;
-    const bool pair = p.pair != 0;
-    p.stg_sw = g.bits == 4 ? packed_sw_mask(pl.bkp) : 0;
-    s = encode_x_map(d, g, x, pl.bkp,
-                     pair ? CU_TENSOR_MAP_SWIZZLE_NONE : (g.bits == 4 ? packed_swizzle(pl.bkp) : swizzle_for(pl.BK)),
-                     &xm);
+qc_status qconv_plan_set(const qconv_desc *d, const qconv_plan *choice) {
+    Exec ex;
+    qc_status s = derive_exec(d, true, &ex);
     if (s != QC_OK) return s;
-    s = encode_w_map(d, g, w8, pair ? 16 : pl.BK, pl.BN,
-                     pair ? CU_TENSOR_MAP_SWIZZLE_NONE : swizzle_for(pl.BK), &wm);
-    if (s != QC_OK) return s;
+    const std::string key = desc_key(d);
+    std::lock_guard<std::mutex> lk(g_plan_mu);
+    if (!choice) {
+        g_plans.erase(key);
+        return QC_OK;
+    }
+    Choice c;
+    c.kernel = choice->kernel;
+    c.bn = choice->bn;
+    Plan pl;
+    if (c.kernel != QC_KERNEL_AUTO && !resolve(ex, c, &pl)) return QC_ERR_UNSUPPORTED;
+    g_plans[key] = c;
+    return QC_OK;
+}
 
-    alignas(64) CUtensorMap ym;
-    std::memset(&ym, 0, sizeof(ym));
-    if (p.y_tma) {
-        s = encode_y_map(d, g, y, p.y_gw, &ym);
-        if (s != QC_OK) return s;
+void qconv_plan_clear(void) {
+    std::lock_guard<std::mutex> lk(g_plan_mu);
+    g_plans.clear();
+}
+
+int32_t qconv_plan_candidates(const qconv_desc *d, qconv_plan *out, int32_t cap) {
+    Exec ex;
+    if (derive_exec(d, true, &ex) != QC_OK) return 0;
+    const std::vector<Choice> cs = candidates(ex);
+    for (int32_t i = 0; i < static_cast<int32_t>(cs.size()) && i < cap && out; ++i) {
+        Plan pl;
+        resolve(ex, cs[i], &pl);
+        fill_plan_out(ex, pl, &out[i]);
     }
-    const bool is4 = g.bits == 4;
-    {
-        Plan p2;
-        if (make_plan2(d, g, pl, &p2)) {
-            p2.cp.bias = bias; p2.cp.mult = multiplier; p2.cp.shift = shift; p2.cp.y = y;
-            alignas(64) CUtensorMap wm2;
-            s = encode_w_map(d, g, w8, pl.BK, pl.BN / 2, swizzle_for(pl.BK), &wm2);
-            if (s != QC_OK) return s;
-            switch (d->y_t) {
-                case QC_U8: return is4 ? launch_fwd2<true, qc::OUT_U8>(p2, xm, wm2, ym, st) : launch_fwd2<false, qc::OUT_U8>(p2, xm, wm2, ym, st);
-                case QC_S8: return is4 ? launch_fwd2<true, qc::OUT_S8>(p2, xm, wm2, ym, st) : launch_fwd2<false, qc::OUT_S8>(p2, xm, wm2, ym, st);
-                case QC_U4: return is4 ? launch_fwd2<true, qc::OUT_U4>(p2, xm, wm2, ym, st) : launch_fwd2<false, qc::OUT_U4>(p2, xm, wm2, ym, st);
-                case QC_S4: return is4 ? launch_fwd2<true, qc::OUT_S4>(p2, xm, wm2, ym, st) : launch_fwd2<false, qc::OUT_S4>(p2, xm, wm2, ym, st);
-                default: break;
-            }
+    return static_cast<int32_t>(cs.size());
+}
+
+qc_status qconv_autotune(const qconv_desc *d, const void *x, const void *w, const int32_t *bias,
+                         const int32_t *multiplier, const int32_t *shift, void *y, void *workspace,
+                         size_t ws_bytes, void *stream, int32_t iters, qconv_plan *best, float *best_us) {
+    Exec ex;
+    qc_status s = derive_exec(d, false, &ex);
+    if (s != QC_OK) return s;
+    if (iters < 1) return QC_ERR_INVALID_ARG;
+    const std::vector<Choice> cs = candidates(ex);
+    if (cs.empty()) return QC_ERR_UNSUPPORTED;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    cudaEvent_t e0, e1;
+    if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess) return cuda_fail(cudaGetLastError());
+    float best_t = 0.0f;
+    int best_i = -1;
+    for (size_t i = 0; i < cs.size(); ++i) {
+        g_forced = true;
+        g_force = cs[i];
+        s = qconv2d_forward(d, x, w, bias, multiplier, shift, y, workspace, ws_bytes, stream);   // warm-up
+        if (s == QC_OK) {
+            cudaEventRecord(e0, st);
+            for (int it = 0; it < iters && s == QC_OK; ++it)
+                s = qconv2d_forward(d, x, w, bias, multiplier, shift, y, workspace, ws_bytes, stream);
+            cudaEventRecord(e1, st);
         }
+        g_forced = false;
+        if (s != QC_OK) break;
+        cudaError_t err = cudaEventSynchronize(e1);
+        if (err != cudaSuccess) { s = cuda_fail(err); break; }
+        float ms = 0.0f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        const float us = 1000.0f * ms / static_cast<float>(iters);
+        if (best_i < 0 || us < best_t) { best_t = us; best_i = static_cast<int>(i); }
     }
-    switch (d->y_t) {
-        case QC_S32: return is4 ? launch_conv<true, qc::OUT_S32>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_S32>(pl, xm, wm, ym, st);
-        case QC_U8: return is4 ? launch_conv<true, qc::OUT_U8>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_U8>(pl, xm, wm, ym, st);
-        case QC_S8: return is4 ? launch_conv<true, qc::OUT_S8>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_S8>(pl, xm, wm, ym, st);
-        case QC_U4: return is4 ? launch_conv<true, qc::OUT_U4>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_U4>(pl, xm, wm, ym, st);
-        case QC_S4: return is4 ? launch_conv<true, qc::OUT_S4>(pl, xm, wm, ym, st) : launch_conv<false, qc::OUT_S4>(pl, xm, wm, ym, st);
+    g_forced = false;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (s != QC_OK) return s;
+    qconv_plan chosen;
+    std::memset(&chosen, 0, sizeof(chosen));
+    chosen.kernel = cs[best_i].kernel;
+    chosen.bn = cs[best_i].bn;
+    s = qconv_plan_set(d, &chosen);
+    if (s != QC_OK) return s;
+    if (best) {
+        Plan pl;
+        resolve(ex, cs[best_i], &pl);
+        fill_plan_out(ex, pl, best);
     }
-    return QC_ERR_INVALID_ARG;
+    if (best_us) *best_us = best_t;
+    return QC_OK;
 }
 
 // ------------------------------------------------------------------ space-to-depth stem
-static int32_t s2d_channels(int32_t c) {
-    const int32_t c4 = 4 * c;
-    return c4 <= 16 ? 16 : (c4 + 31) / 32 * 32;
-}
-static qc_dtype byte_container(qc_dtype t) {
-    return (t == QC_U4 || t == QC_U8) ? QC_U8 : QC_S8;
-}
-
 qc_status qconv_s2d_desc(const qconv_desc *d, qconv_desc *out) {
     if (!d) return QC_ERR_INVALID_ARG;
     // the original activations are float (quantized by qconv_quantize_pack_s2d), so an odd c
@@ -1173,26 +1418,14 @@ qc_status qconv_s2d_desc(const qconv_desc *d, qconv_desc *out) {
     qconv_desc dv = *d;
     dv.x_t = byte_container(d->x_t);
     Geometry g;
-    qc_status s = validate_desc(&dv, &g);
+    qc_status s = validate_desc(&dv, &g, true);
     if (s != QC_OK) return s;
     if (!is_int_input(d->x_t) || d->x_zero < dtype_min(d->x_t) || d->x_zero > dtype_max(d->x_t))
         return QC_ERR_INVALID_ARG;
     if (!out) return QC_ERR_INVALID_ARG;
-    if (d->stride_h != 2 || d->stride_w != 2 || d->dil_h != 1 || d->dil_w != 1)
-        return QC_ERR_UNSUPPORTED;
-    qconv_desc o = *d;
-    o.r = (d->r + 1) / 2;
-    o.s = (d->s + 1) / 2;
-    o.h = g.P + o.r - 1;
-    o.w = g.Q + o.s - 1;
-    o.c = s2d_channels(d->c);
-    o.stride_h = o.stride_w = 1;
-    o.pad_h = o.pad_w = 0;
-    o.dil_h = o.dil_w = 1;
-    o.x_t = byte_container(d->x_t);
-    o.w_t = byte_container(d->w_t);
-    o.w_prepared = 1;
-    *out = o;
+    if (d->stride_h != 2 || d->stride_w != 2 || d->dil_h != 1 || d->dil_w != 1) return QC_ERR_UNSUPPORTED;
+    if (d->w_zero) return QC_ERR_UNSUPPORTED;
+    *out = s2d_of(d, g);
     return QC_OK;
 }
 
@@ -1256,7 +1489,7 @@ qc_status qconv_debug_im2col_tile(const qconv_desc *d, const void *x, int64_t m0
                                   int32_t s_, int32_t c_byte, int32_t box_bytes, void *out,
                                   void *stream) {
     Geometry g;
-    qc_status s = validate_desc(d, &g);
+    qc_status s = validate_desc(d, &g, true);
     if (s != QC_OK) return s;
     if (!x || !out || m0 < 0 || m0 >= g.M || r < 0 || r >= d->r || s_ < 0 || s_ >= d->s ||
         box_bytes < 16 || box_bytes > 256 || box_bytes % 16 || c_byte < 0 ||

@@ -13,7 +13,7 @@
 // saturating pack into the pair's byte (4-bit) or 16-bit word (8-bit) of an NHWC row,
 // staged (swizzled) in shared memory and written by TMA stores.
 #pragma once
-#include "conv_fwd.cuh"
+#include "epilogue.cuh"
 
 namespace qc {
 
@@ -22,8 +22,9 @@ struct TChan {          // per-channel constants held in registers by the epilog
     int32_t m, sh, b, k, vlim, n;
 };
 
-// Re-quantize one accumulator of one channel (Eq.(3)-(4)); `mode` is warp
-// uniform: 0 fast (shift 33..52), 1 mid (shift 20..50), 2 general (see conv_fwd.cuh EpiCol).
+// Re-quantize one accumulator of one channel; `mode` is warp uniform:
+// 0 fast (shift 33..52), 1 mid (shift 20..50, |m| >= 2^30 or m == 0), 2 general (either
+// rounding, see epilogue.cuh EpiCol).
 template <int MODE>
 __device__ __forceinline__ int32_t t_requant(const ConvParams &p, const TChan &c, uint32_t acc) {
     int32_t y;
@@ -36,9 +37,15 @@ __device__ __forceinline__ int32_t t_requant(const ConvParams &p, const TChan &c
     } else {
         const int64_t lo64 = static_cast<int64_t>(p.clamp_lo) - p.y_zero;
         const int64_t hi64 = static_cast<int64_t>(p.clamp_hi) - p.y_zero;
-        const int64_t prod = static_cast<int64_t>((static_cast<int32_t>(acc) >> p.acc_lg) + c.b) * c.m +
-                             (static_cast<int64_t>(1) << (c.n - 1));
-        int64_t t = prod >> c.n;
+        const int32_t x = static_cast<int32_t>(static_cast<uint32_t>(static_cast<int32_t>(acc) >> p.acc_lg) +
+                                               static_cast<uint32_t>(c.b));
+        int64_t t;
+        if (p.round_tfl) {
+            t = requant_tflite(x, c.m, c.n);
+        } else {
+            const int64_t prod = static_cast<int64_t>(x) * c.m + (static_cast<int64_t>(1) << (c.n - 1));
+            t = prod >> c.n;
+        }
         t = t < lo64 ? lo64 : (t > hi64 ? hi64 : t);
         y = static_cast<int32_t>(t) + p.y_zero;
     }
@@ -95,10 +102,6 @@ __device__ __forceinline__ void t_pairs(const ConvParams &p, const TChan &ce, co
 template <int OUT, int RB, int GMASK>
 __device__ __forceinline__ void t_pairs_mode(const ConvParams &p, int mode, const TChan &ce, const TChan &co,
                                              const uint32_t (&v)[32], uint32_t ystg, int row0, uint32_t boff) {
-    if (p.exp_flags & 16) {                       // debug ablation: TMEM loads only
-        if (v[0] == 0x9e3779b9u && row0 == 12345) asm volatile("trap;");
-        return;
-    }
     if (p.need_clamp) {
         if (mode == 0) t_pairs<OUT, 0, true, RB, GMASK>(p, ce, co, v, ystg, row0, boff);
         else if (mode == 1) t_pairs<OUT, 1, true, RB, GMASK>(p, ce, co, v, ystg, row0, boff);
@@ -131,13 +134,6 @@ __device__ __forceinline__ void t_chan_mid(const ConvParams &p, TChan &c, int ne
     c.c64 = static_cast<int64_t>((1 << (T - 33)) + p.y_zero * (1 << (T - 32))) << 32;
 }
 
-// 16 epilogue warps (4 per SMSP: the re-quantization is latency- not issue-bound), then the
-// 4 converter warps (4-bit).
-constexpr int kTEpiWarps = 16;
-constexpr int kTProducers = 2;        // TMA issuers: lane 0 of warps 0 and 3 (warp 2: output storer)
-constexpr int kTWarpCvt0 = kWarpEpi0 + kTEpiWarps;
-constexpr int kTThreads8 = 32 * kTWarpCvt0;
-constexpr int kTThreads4 = 32 * (kTWarpCvt0 + kNumCvtWarps);
 
 template <bool IS4, int OUT, bool M64>
 __global__ void __launch_bounds__(IS4 ? kTThreads4 : kTThreads8, 1)
@@ -201,8 +197,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 const int m0 = (tile / p.n_tiles_n) * BNp;
                 const int c0 = (tile % p.n_tiles_n) * BMc;
                 mbar_wait(&sfull[b], static_cast<uint32_t>(it >> 1) & 1u);
-                if (!(p.exp_flags & 128))
-                    tma_store_2d(&ymap, smem + p.off_ystg + b * p.ystg_bytes, c0 * (kInt4 ? 4 : 8) / 8, m0);
+                tma_store_2d(&ymap, smem + p.off_ystg + b * p.ystg_bytes, c0 * (kInt4 ? 4 : 8) / 8, m0);
                 bulk_commit();
                 bulk_wait_read<1>();                 // the store from buffer b^1 has read its smem
                 if (it > 0) mbar_arrive(&sfree[b ^ 1]);
@@ -272,13 +267,11 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                     if (ksteps == 4) {
 #pragma unroll
                         for (int k = 0; k < 4; ++k)
-                            if (!(p.exp_flags & 4) || (kb | k) == 0)
-                                mma_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
+                            mma_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
                                                (kb | k) != 0 ? 1u : 0u);
                     } else {
                         for (int k = 0; k < ksteps; ++k)
-                            if (!(p.exp_flags & 4) || (kb | k) == 0)
-                                mma_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
+                            mma_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
                                                (kb | k) != 0 ? 1u : 0u);
                     }
                     mma_commit_warp(&empty[stage]);
@@ -321,8 +314,9 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 t_chan_params(p, ko, ko < p.K, co, neo, bo);
                 const unsigned act = 0xffffffffu;
                 const bool all_fast = __ballot_sync(act, be && bo && nee >= 33 && nee <= 52 && neo >= 33 && neo <= 52) == act;
-                const bool all_mid = __ballot_sync(act, be && bo && nee >= 20 && nee <= 50 && neo >= 20 && neo <= 50) == act;
-                mode = all_fast ? 0 : (all_mid ? 1 : 2);
+                const bool all_mid = __ballot_sync(act, be && bo && nee >= 20 && nee <= 50 && neo >= 20 && neo <= 50 &&
+                                                            mid_multiplier_ok(ce.m) && mid_multiplier_ok(co.m)) == act;
+                mode = p.round_tfl ? 2 : (all_fast ? 0 : (all_mid ? 1 : 2));
                 if (mode == 1) {
                     const int T = max(33, __reduce_max_sync(act, max(nee, neo)));
                     t_chan_mid(p, ce, nee, T);
@@ -372,7 +366,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 if (ct == 0) trace_ev(p, 8, g);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
-                if (!(p.exp_flags & 8)) widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
+                widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
                 if (ct == 0) trace_ev(p, 10, g);
                 fence_proxy_async_smem();
                 __syncwarp();

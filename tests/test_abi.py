@@ -74,10 +74,18 @@ def test_forward_host_validation():
     assert _fwd(qc.make_desc(**good, x_t=qc.QC_S32)) == 1                   # bad input dtype
     assert _fwd(qc.make_desc(**good, clamp_lo=10, clamp_hi=5)) == 1
     assert _fwd(qc.make_desc(**good, y_zero=300)) == 1
+    assert _fwd(qc.make_desc(**good, rounding=2)) == 1
+    assert _fwd(qc.make_desc(**good, y_t=qc.QC_F32_OUT)) == 1               # float: dequant call
     assert _fwd(qc.make_desc(**good), x=None) == 1
     assert _fwd(qc.make_desc(**good), m=None) == 1                          # requant ptrs needed
-    assert _fwd(qc.make_desc(**{**good, "c": 48})) == 2                     # UNSUPPORTED (C%32)
-    assert _fwd(qc.make_desc(**good, x_t=qc.QC_U4, w_t=qc.QC_S8)) == 2      # mixed widths
+    assert _fwd(qc.make_desc(**{**good, "c": 3}, x_t=qc.QC_U4, w_t=qc.QC_S4)) == 1  # odd 4-bit rows
+    # channel counts the kernels do not take directly are rearranged into the workspace
+    d48 = qc.make_desc(**{**good, "c": 48})
+    assert qc.qconv2d_workspace_size(d48) == 64 * 9 * 64 + 8 * 8 * 64      # padded w + activations
+    assert qc.qconv_prepared_weight_bytes(d48) == 64 * 9 * 64
+    assert _fwd(d48) == 5                                                   # WORKSPACE
+    assert qc.qconv_debug_plan(d48)["prologue"] == 1 | 2
+    assert _fwd(qc.make_desc(**good, x_t=qc.QC_U4, w_t=qc.QC_S8)) == 2      # A4W8
     assert _fwd(qc.make_desc(**{**good, "k": 63}, x_t=qc.QC_U4, w_t=qc.QC_S4,
                              y_t=qc.QC_U4)) == 2                            # odd K, 4-bit out
     assert _fwd(qc.make_desc(**{**good, "stride": 9})) == 2
@@ -92,6 +100,42 @@ def test_forward_host_validation():
     d4.w_prepared = 1
     assert qc.qconv2d_workspace_size(d4) == 0
     assert qc.qconv_prepared_weight_bytes(d4) == 64 * 9 * 64 + 4 * 64
+    # A8W4: 4-bit weights widened to int8 (no weight sums)
+    da = qc.make_desc(**good, x_t=qc.QC_U8, w_t=qc.QC_S4)
+    assert qc.qconv_prepared_weight_bytes(da) == 64 * 9 * 64
+    assert qc.qconv2d_workspace_size(da) == 64 * 9 * 64
+    # weight zero points: per-pixel activation sums in the workspace, im2col kernel
+    dz = qc.make_desc(**good, w_zero=FAKE)
+    assert qc.qconv2d_workspace_size(dz) == 256 + 256
+    assert qc.qconv_debug_plan(dz)["kernel_name"] == "im2col"
+    assert _fwd(dz) == 5
+
+
+def test_plans_on_the_host():
+    """Kernel choice, candidates and the plan cache need no GPU (no launch)."""
+    qc.qconv_plan_clear()
+    d = qc.make_desc(256, 14, 14, 256, 256, 3, 3, pad=1, x_t=qc.QC_U4, w_t=qc.QC_S4,
+                     y_t=qc.QC_U4, w_prepared=1)
+    assert qc.qconv_debug_plan(d)["kernel_name"] == "pair"
+    cands = qc.qconv_plan_candidates(d)
+    names = {(c["kernel_name"], c["bn"]) for c in cands}
+    assert ("im2col", 256) in names and ("pair", 256) in names and ("im2col", 64) in names
+    qc.qconv_plan_set(d, qc.QC_KERNEL_IM2COL, 128)
+    p = qc.qconv_debug_plan(d)
+    assert (p["kernel_name"], p["bn"]) == ("im2col", 128)
+    with pytest.raises(qc.QConvError):
+        qc.qconv_plan_set(d, qc.QC_KERNEL_CHANNEL, 128)                      # 3x3: ineligible
+    qc.qconv_plan_set(d, None)
+    assert qc.qconv_debug_plan(d)["kernel_name"] == "pair"
+    # 1x1 -> channel-major; stem in s2d form -> halo; int32 output -> im2col
+    d1 = qc.make_desc(32, 56, 56, 64, 256, 1, 1, x_t=qc.QC_U4, w_t=qc.QC_S4, y_t=qc.QC_S4,
+                      w_prepared=1)
+    assert qc.qconv_debug_plan(d1)["kernel_name"] == "channel"
+    stem = qc.make_desc(8, 224, 224, 3, 64, 7, 7, stride=2, pad=3, w_prepared=1)
+    ps = qc.qconv_debug_plan(stem)
+    assert ps["kernel_name"] == "halo" and ps["prologue"] == 2
+    d32 = qc.make_desc(2, 9, 9, 64, 48, 3, 3, pad=1, y_t=qc.QC_S32)
+    assert qc.qconv_debug_plan(d32)["kernel_name"] == "im2col"
 
 
 def test_quantize_host_validation():

@@ -139,17 +139,29 @@ def test_cta_pair_8bit_3x3_full_tiles(cs):
         np.testing.assert_array_equal(got[img:img + 1], ref, err_msg=f"{cs.name} img {img}")
 
 
-def test_cta_pair_forced_every_eligible_layer():
-    """QC_CTA2=1 (read once per process) forces the CTA-pair kernel onto every eligible
-    im2col layer, 4-bit included: run the small-shape and ResNet-50 parity tests that way in
-    a child process."""
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    env = dict(os.environ, QC_CTA2="1")
-    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu",
-                        os.path.join(root, "tests", "test_gpu_parity.py"), "-k",
-                        "small_shapes or resnet50_all or shift_ranges or signed_activations"],
-                       cwd=root, env=env, capture_output=True, text=True, timeout=600)
-    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+@pytest.mark.parametrize("bits", [8, 4])
+def test_cta_pair_forced_every_eligible_layer(bits):
+    """Force the CTA-pair kernel (through the plan API) onto every ResNet-50 layer at batch 2
+    where it is eligible, 4-bit included, with the widest N tile it takes."""
+    from workloads import resnet50_convs, stored_channels
+    n_forced = 0
+    for i, cs in enumerate(resnet50_convs(2)):
+        li = make_layer_inputs(cs, bits, seed=4000 + i, relu=True, c_store=stored_channels(cs, bits))
+        d = qc.make_desc(cs.n, cs.h, cs.w, li.x_codes.shape[-1], cs.k, cs.r, cs.s, stride=cs.stride,
+                         pad=cs.pad, x_t=li.x_t, w_t=li.w_t, y_t=li.y_t, clamp_lo=li.clamp_lo,
+                         clamp_hi=li.clamp_hi)
+        pairs = [c for c in qc.qconv_plan_candidates(d) if c["kernel"] == qc.QC_KERNEL_PAIR]
+        if not pairs:
+            continue
+        bn = max(c["bn"] for c in pairs)
+        m, n = oracle.requant_params(li.s_x, li.s_w, li.s_y)
+        qc.qconv_plan_set(d, qc.QC_KERNEL_PAIR, bn)
+        try:
+            assert qc.qconv_debug_plan(d)["kernel"] == qc.QC_KERNEL_PAIR
+            got = _run(li, m, n)
+        finally:
+            qc.qconv_plan_set(d, None)
+        ref = oracle.conv2d_layer(li, mult=m, shift=n)
+        np.testing.assert_array_equal(got, ref, err_msg=f"{cs.name} pair bn={bn}")
+        n_forced += 1
+    assert n_forced >= 20

@@ -267,8 +267,6 @@ def test_resnet50_batch32_sampled(bits):
 
 def test_vgg16_batch2_8bit():
     for i, cs in enumerate(vgg16_convs(2)):
-        if cs.c == 3:
-            continue
         _check_layer(make_layer_inputs(cs, 8, seed=3000 + i))
 
 

@@ -337,3 +337,20 @@ def layer_seed(index: int) -> int:
 def float_image(rng: np.random.Generator, shape) -> np.ndarray:
     """fp32 activations ReLU(N(0,1)) (C2 recipe)."""
     return np.maximum(rng.normal(0.0, 1.0, size=shape), 0.0).astype(np.float32)
+
+
+def device_post_relu_codes(shape, bits: int, seed: int, device):
+    """Packed post-ReLU activation codes drawn on the GPU with a seeded torch generator (same
+    recipe as post_relu_codes: ~50 % zeros, rest round(|N(0, 40/255 * qmax)|) clipped) -- for
+    bench-sized layers whose inputs are too large to draw on the host.  Returns a uint8 tensor
+    [..., C * bits / 8] in the boundary's byte layout (Z7 nibble order)."""
+    import torch
+    g = torch.Generator(device=device)
+    g.manual_seed(int(seed))
+    qmax = (1 << bits) - 1
+    v = torch.randn(shape, generator=g, device=device).abs_().mul_(40 / 255 * qmax).round_()
+    v[torch.rand(shape, generator=g, device=device) < 0.5] = 0
+    codes = v.clamp_(0, qmax).to(torch.uint8)
+    if bits == 4:
+        return (codes[..., 0::2] | (codes[..., 1::2] << 4)).contiguous()
+    return codes
