@@ -809,6 +809,7 @@ qc_status encode_halo_maps(const qconv_desc *d, const Geometry &g, const qc::Con
 // excludes them (the plan API can still choose it).
 bool make_trans_plan(const qconv_desc *d, const Geometry &g, int bmc_req, bool chosen, Plan *pl) {
     if (d->r != 1 || d->s != 1 || d->x_zero != 0 || !is_packed_out(d->y_t)) return false;
+    if (d->rounding == QC_ROUND_TFLITE) return false;   // kept out of its epilogue (register budget)
     if (d->c % 32 || d->k % 64) return false;
     const bool is4 = g.bits == 4;
     if (!chosen && is4 && d->c > 512) return false;

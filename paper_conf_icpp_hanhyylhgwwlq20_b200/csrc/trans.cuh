@@ -23,8 +23,8 @@ struct TChan {          // per-channel constants held in registers by the epilog
 };
 
 // Re-quantize one accumulator of one channel; `mode` is warp uniform:
-// 0 fast (shift 33..52), 1 mid (shift 20..50, |m| >= 2^30 or m == 0), 2 general (either
-// rounding, see epilogue.cuh EpiCol).
+// 0 fast (shift 33..52), 1 mid (shift 20..50, |m| >= 2^30 or m == 0), 2 general (see
+// epilogue.cuh EpiCol).  The TFLite rounding is not taken here (qconv.cu plans it elsewhere).
 template <int MODE>
 __device__ __forceinline__ int32_t t_requant(const ConvParams &p, const TChan &c, uint32_t acc) {
     int32_t y;
@@ -39,13 +39,8 @@ __device__ __forceinline__ int32_t t_requant(const ConvParams &p, const TChan &c
         const int64_t hi64 = static_cast<int64_t>(p.clamp_hi) - p.y_zero;
         const int32_t x = static_cast<int32_t>(static_cast<uint32_t>(static_cast<int32_t>(acc) >> p.acc_lg) +
                                                static_cast<uint32_t>(c.b));
-        int64_t t;
-        if (p.round_tfl) {
-            t = requant_tflite(x, c.m, c.n);
-        } else {
-            const int64_t prod = static_cast<int64_t>(x) * c.m + (static_cast<int64_t>(1) << (c.n - 1));
-            t = prod >> c.n;
-        }
+        const int64_t prod = static_cast<int64_t>(x) * c.m + (static_cast<int64_t>(1) << (c.n - 1));
+        int64_t t = prod >> c.n;
         t = t < lo64 ? lo64 : (t > hi64 ? hi64 : t);
         y = static_cast<int32_t>(t) + p.y_zero;
     }
@@ -316,7 +311,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 const bool all_fast = __ballot_sync(act, be && bo && nee >= 33 && nee <= 52 && neo >= 33 && neo <= 52) == act;
                 const bool all_mid = __ballot_sync(act, be && bo && nee >= 20 && nee <= 50 && neo >= 20 && neo <= 50 &&
                                                             mid_multiplier_ok(ce.m) && mid_multiplier_ok(co.m)) == act;
-                mode = p.round_tfl ? 2 : (all_fast ? 0 : (all_mid ? 1 : 2));
+                mode = all_fast ? 0 : (all_mid ? 1 : 2);
                 if (mode == 1) {
                     const int T = max(33, __reduce_max_sync(act, max(nee, neo)));
                     t_chan_mid(p, ce, nee, T);

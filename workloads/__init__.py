@@ -354,3 +354,33 @@ def device_post_relu_codes(shape, bits: int, seed: int, device):
     if bits == 4:
         return (codes[..., 0::2] | (codes[..., 1::2] << 4)).contiguous()
     return codes
+
+
+def densenet121_convs(batch: int) -> List[ConvShape]:
+    """The 120 conv layers of DenseNet-121 (growth 32, bottleneck 4 x 32, blocks 6/12/24/16,
+    compression 0.5) in network order -- the paper's second GPU workload (Fig.17:
+    "input size for conv15 ... is 1 x 14 x 14 x 736").  The stem is 7x7/s2 over C = 3."""
+    out = [ConvShape("dn_conv0", batch, 224, 224, 3, 64, 7, 7, 2, 3)]
+    c, hw = 64, 56
+    for b, nl in enumerate((6, 12, 24, 16)):
+        for i in range(nl):
+            cin = c + 32 * i
+            out.append(ConvShape(f"dn_b{b + 1}_l{i + 1}_1x1", batch, hw, hw, cin, 128, 1, 1))
+            out.append(ConvShape(f"dn_b{b + 1}_l{i + 1}_3x3", batch, hw, hw, 128, 32, 3, 3, 1, 1))
+        c += 32 * nl
+        if b < 3:
+            out.append(ConvShape(f"dn_t{b + 1}", batch, hw, hw, c, c // 2, 1, 1))
+            c //= 2
+            hw //= 2
+    return out
+
+
+def densenet121_unique(batch: int = 1) -> List[ConvShape]:
+    """Unique DenseNet-121 conv shapes (first occurrence order), stem excluded."""
+    seen, out = set(), []
+    for cs in densenet121_convs(batch)[1:]:
+        key = (cs.h, cs.w, cs.c, cs.k, cs.r, cs.s, cs.stride, cs.pad)
+        if key not in seen:
+            seen.add(key)
+            out.append(cs)
+    return out
