@@ -83,11 +83,12 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
             const uint32_t tx = static_cast<uint32_t>(kBM * (p.pair ? 32 : p.bkp) + p.BN * p.BK);
             int g = 0;                                              // CTA-local K-stage counter
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
-                const int m0 = (tile / p.n_tiles_n) * kBM;
-                const int n0 = (tile % p.n_tiles_n) * p.BN;
-                const int img = m0 / p.PQ;
+                const int mt = p.fd_ntn.div(tile);
+                const int m0 = mt * kBM;
+                const int n0 = (tile - mt * p.n_tiles_n) * p.BN;
+                const int img = p.fd_pq.div(m0);
                 const int rem = m0 - img * p.PQ;
-                const int p0 = rem / p.Q;
+                const int p0 = p.fd_q.div(rem);
                 const int q0 = rem - p0 * p.Q;
                 const int wb = q0 * p.stride_w - p.pad_w;
                 const int hb = p0 * p.stride_h - p.pad_h;
@@ -101,9 +102,9 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                     if (p.pair) {
                         const int RS = p.R * p.S;
                         const int t0 = 2 * kb, t1 = t0 + 1;
-                        const int r0 = t0 / p.S, s0 = t0 - r0 * p.S;
+                        const int r0 = p.fd_s.div(t0), s0 = t0 - r0 * p.S;
                         int r1 = r0, s1 = s0, kg1 = RS * 16;        // odd tail: B slot OOB -> 0
-                        if (t1 < RS) { r1 = t1 / p.S; s1 = t1 - r1 * p.S; kg1 = t1 * 16; }
+                        if (t1 < RS) { r1 = p.fd_s.div(t1); s1 = t1 - r1 * p.S; kg1 = t1 * 16; }
                         uint8_t *adst = smem + p.off_a + stage * p.a_stage_bytes;
                         uint8_t *bdst = smem + p.off_b + stage * p.b_stage_bytes;
                         if (leader) tma_load_im2col_4d(adst, &xmap, &full[stage], 0, wb, hb, img,
@@ -113,9 +114,9 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                         if (leader) tma_load_2d(bdst, &wmap, &full[stage], t0 * 16, n0);
                         if (leader) tma_load_2d(bdst + p.BN * 16, &wmap, &full[stage], kg1, n0);
                     } else {
-                        const int r = kb / taps_per_r;
+                        const int r = p.fd_tpr.div(kb);
                         const int rem2 = kb - r * taps_per_r;
-                        const int s = rem2 / p.chunks;
+                        const int s = p.fd_chunks.div(rem2);
                         const int ch = rem2 - s * p.chunks;
                         uint8_t *adst = IS4 ? smem + p.off_stg + stage * p.stg_stage_bytes
                                             : smem + p.off_a + stage * p.a_stage_bytes;
@@ -202,8 +203,9 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
-            const int m0 = (tile / p.n_tiles_n) * kBM;
-            const int n0 = (tile % p.n_tiles_n) * p.BN;
+            const int mt = p.fd_ntn.div(tile);
+            const int m0 = mt * kBM;
+            const int n0 = (tile - mt * p.n_tiles_n) * p.BN;
             if (n0 != cached_n0) {
                 fill_epilogue_params<OUT>(p, par, chunk_info, n0, ew, lane, force_general);
                 cached_n0 = n0;

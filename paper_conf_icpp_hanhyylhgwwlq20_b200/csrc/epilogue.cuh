@@ -27,6 +27,7 @@ constexpr int kNumEpiWarps = 8;
 constexpr int kWarpCvt0 = 12;        // warps 12..15: int4 -> int8 converters (4-bit only)
 constexpr int kNumCvtWarps = 4;
 
+constexpr int kMaxYstg = 4;          // halo / channel-major kernels: output staging buffers (max)
 constexpr int kHaloMaxMMA = 18;      // halo kernel: 3x3 taps x 2 plane pairs (C = 64), or the 4x4/2 stem pairs
 // channel-major kernel: 16 epilogue warps (4 per SMSP: the re-quantization is latency- not
 // issue-bound), then the 4 converter warps (4-bit)
@@ -44,6 +45,27 @@ template <int OUT> struct OutTraits {
     static constexpr bool kFloat = OUT == OUT_F32 || OUT == OUT_BF16;
 };
 
+// n / d by multiply-high for 0 <= n < 2^31, 1 <= d < 2^31: with l = ceil(log2 d) and
+// p = 31 + l, mul = ceil(2^p / d) < 2^32 and n / d = umulhi(n, mul) >> (p - 32) (the round-up
+// multiplier method; the producers' per-tile / per-stage index math is on the critical path of
+// the TMA issue loop, where an integer division costs a long dependent chain).
+struct FastDiv {
+    uint32_t d, mul, shr;
+    __device__ __forceinline__ int div(int n) const {
+        return d == 1u ? n : static_cast<int>(__umulhi(static_cast<uint32_t>(n), mul) >> shr);
+    }
+};
+inline FastDiv make_fastdiv(uint32_t d) {
+    FastDiv f;
+    f.d = d;
+    if (d <= 1u) { f.d = 1u; f.mul = 0u; f.shr = 0u; return f; }
+    const uint32_t l = 32u - static_cast<uint32_t>(__builtin_clz(d - 1u));
+    const uint64_t p = 31u + l;
+    f.mul = static_cast<uint32_t>(((uint64_t(1) << p) + d - 1u) / d);
+    f.shr = static_cast<uint32_t>(p - 32u);
+    return f;
+}
+
 struct ConvParams {
     // GEMM geometry
     int32_t M, P, Q, PQ, K;
@@ -55,6 +77,12 @@ struct ConvParams {
     int32_t y_tma;                    // epilogue stages the whole output tile in smem -> TMA store
     uint32_t off_ystg;                // staging: 2 buffers x n_ygroups x [128 rows x y_gw bytes], swizzled
     uint32_t ystg_bytes;              // one staging buffer
+    int32_t n_ystg;                   // halo / channel-major: staging buffers in the ring (2..4)
+    int32_t n_wide;                   // channel-major 4-bit: widened operand slots (2..4)
+    int32_t b_res;                    // channel-major: the CTA's weights resident at off_bres
+    const uint8_t *x_lin;             // channel-major 4-bit, 1x1/s1/p0, one K chunk: activations read
+                                      // as one contiguous bulk copy per tile (else null: im2col TMA)
+    int32_t x_row_bytes;              // packed bytes per pixel (x_lin)
     int32_t y_gw, y_gmask, n_ygroups; // staging group width (32/64/128 B), swizzle mask, count
     int32_t cvt_shift;                // log2(16-byte packed chunks per pixel) for the converter
     int32_t need_clamp;               // clamp range narrower than the output dtype range
@@ -89,11 +117,13 @@ struct ConvParams {
     const int32_t *wsum;              // [K] sum_{r,s,c} w (true values) when x_sgn4, else null
     void *y;
     int64_t y_row_bytes;
+    // fast divisions by P*Q, Q, n_tiles_n, S*chunks, chunks, S, tiles_per_img (set at launch)
+    FastDiv fd_pq, fd_q, fd_ntn, fd_tpr, fd_chunks, fd_s, fd_tpi;
 };
 
 #ifdef QC_DEBUG
 __device__ __forceinline__ void trace_ev(const ConvParams &p, int ev, int seq) {
-    if (p.trace != nullptr && blockIdx.x == 0 && seq < 1024) p.trace[ev * 1024 + seq] = globaltimer_ns();
+    if (p.trace != nullptr && blockIdx.x == 0 && seq < 1024) p.trace[ev * 1024 + seq] = clock64();   // SM cycles
 }
 #else
 __device__ __forceinline__ void trace_ev(const ConvParams &, int, int) {}

@@ -176,11 +176,12 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
             const uint32_t tx = static_cast<uint32_t>(kBM * p.bkp + half_bn * p.BK);
             int g = 0;
             for (int tile = pair; tile < p.num_tiles; tile += npairs) {
-                const int m0 = (tile / p.n_tiles_n) * (2 * kBM) + static_cast<int>(rank) * kBM;
-                const int n0 = (tile % p.n_tiles_n) * p.BN + static_cast<int>(rank) * half_bn;
-                const int img = m0 / p.PQ;
+                const int mt = p.fd_ntn.div(tile);
+                const int m0 = mt * (2 * kBM) + static_cast<int>(rank) * kBM;
+                const int n0 = (tile - mt * p.n_tiles_n) * p.BN + static_cast<int>(rank) * half_bn;
+                const int img = p.fd_pq.div(m0);
                 const int rem = m0 - img * p.PQ;
-                const int p0 = rem / p.Q;
+                const int p0 = p.fd_q.div(rem);
                 const int q0 = rem - p0 * p.Q;
                 const int wb = q0 * p.stride_w - p.pad_w;
                 const int hb = p0 * p.stride_h - p.pad_h;
@@ -190,9 +191,9 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                     const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
                     mbar_wait(&empty[stage], phase ^ 1u);
                     trace_ev2(p, rank ? 7 : 0, g, rank);
-                    const int r = kb / taps_per_r;
+                    const int r = p.fd_tpr.div(kb);
                     const int rem2 = kb - r * taps_per_r;
-                    const int s = rem2 / p.chunks;
+                    const int s = p.fd_chunks.div(rem2);
                     const int ch = rem2 - s * p.chunks;
                     uint8_t *adst = IS4 ? smem + p.off_stg + stage * p.stg_stage_bytes
                                         : smem + p.off_a + stage * p.a_stage_bytes;
@@ -276,8 +277,9 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
         for (int tile = pair; tile < p.num_tiles; tile += npairs, ++it) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
-            const int m0 = (tile / p.n_tiles_n) * (2 * kBM) + static_cast<int>(rank) * kBM;
-            const int n0 = (tile % p.n_tiles_n) * p.BN;
+            const int mt = p.fd_ntn.div(tile);
+            const int m0 = mt * (2 * kBM) + static_cast<int>(rank) * kBM;
+            const int n0 = (tile - mt * p.n_tiles_n) * p.BN;
             if (n0 != cached_n0) {
                 fill_epilogue_params<OUT>(p, par, chunk_info, n0, ew, lane, false);
                 cached_n0 = n0;

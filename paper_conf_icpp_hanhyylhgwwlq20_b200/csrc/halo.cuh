@@ -40,9 +40,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
     uint64_t *tfull = bars + 3 * NS;        // [2]
     uint64_t *tempty = bars + 3 * NS + 2;   // [2]
     uint64_t *bfull = bars + 3 * NS + 4;    // [1] resident weights landed
-    uint64_t *sfull = bars + 3 * NS + 5;    // [2] epilogue warps -> storer: staging buffer written
-    uint64_t *sfree = bars + 3 * NS + 7;    // [2] storer -> epilogue warps: its TMA store has read it
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 9);
+    uint64_t *sfull = bars + 3 * NS + 5;    // [kMaxYstg] epilogue warps -> storer: staging buffer written
+    uint64_t *sfree = bars + 3 * NS + 5 + kMaxYstg;   // [kMaxYstg] storer -> epilogue warps: store read it
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 5 + 2 * kMaxYstg);
+    const int NB = p.n_ystg;                 // staging buffers
     EpiCol *par = reinterpret_cast<EpiCol *>(smem + p.off_par);
     int4 *chunk_info = reinterpret_cast<int4 *>(smem + p.off_par + 16 * kMaxBN);
 
@@ -59,6 +60,8 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         for (int i = 0; i < 2; ++i) {
             mbar_init(&tfull[i], 1);
             mbar_init(&tempty[i], kNumEpiWarps);
+        }
+        for (int i = 0; i < kMaxYstg; ++i) {
             mbar_init(&sfull[i], kNumEpiWarps);
             mbar_init(&sfree[i], 1);
         }
@@ -78,11 +81,11 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         if (lane == 0) {
             int it = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
-                const int b = it & 1;
-                const int mt = tile / p.n_tiles_n;
-                const int img = mt / p.tiles_per_img;
+                const int b = it % NB;
+                const int mt = p.fd_ntn.div(tile);
+                const int img = p.fd_tpi.div(mt);
                 const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
-                mbar_wait(&sfull[b], static_cast<uint32_t>(it >> 1) & 1u);
+                mbar_wait(&sfull[b], static_cast<uint32_t>(it / NB) & 1u);
                 {
                     constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
                     for (int gi = 0; gi < p.n_ygroups; ++gi)
@@ -90,8 +93,9 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                                      n0 * kBits / 8 + gi * p.y_gw, 0, p0, img);
                 }
                 bulk_commit();
+                // keep two stores in flight: the previous one has read its buffer -> release it
                 bulk_wait_read<1>();
-                if (it > 0) mbar_arrive(&sfree[b ^ 1]);
+                if (it > 0) mbar_arrive(&sfree[(it - 1) % NB]);
                 trace_ev(p, 7, it);
             }
             bulk_wait<0>();
@@ -107,8 +111,8 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             if (leader) tma_load_3d(smem + p.off_bres, &bmap, bfull, 0, n0, 0);
             int g = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
-                const int mt = tile / p.n_tiles_n;
-                const int img = mt / p.tiles_per_img;
+                const int mt = p.fd_ntn.div(tile);
+                const int img = p.fd_tpi.div(mt);
                 const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
                 const int stage = g % NS;
                 const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
@@ -209,8 +213,9 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             tc_fence_after();
             const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
                                    static_cast<uint32_t>(buf * p.BN);
-            mbar_wait(&sfree[it & 1], (static_cast<uint32_t>(it >> 1) & 1u) ^ 1u);
-            const uint32_t ystg_it = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes;
+            const int sb = it % NB;
+            mbar_wait(&sfree[sb], (static_cast<uint32_t>(it / NB) & 1u) ^ 1u);
+            const uint32_t ystg_it = ystg_base + static_cast<uint32_t>(sb) * p.ystg_bytes;
             // TMEM loads double-buffered: chunk ci+2 is in flight while chunk ci is requantized
             uint32_t va[32], vb[32];
             auto process = [&](uint32_t (&v)[32], int ci) {
@@ -251,7 +256,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             __syncwarp();
             if (lane == 0) {
                 mbar_arrive(&tempty[buf]);
-                mbar_arrive(&sfull[it & 1]);
+                mbar_arrive(&sfull[sb]);
             }
             if (ew == 0 && lane == 0) trace_ev(p, 6, it);
         }

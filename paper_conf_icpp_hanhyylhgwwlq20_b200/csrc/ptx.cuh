@@ -86,6 +86,29 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     }
 }
 
+// Wait for a control role (TMA producer, MMA issuer, output storer): the thread is suspended
+// in hardware until the phase completes (suspend-time hint), so a waiting control warp -- which
+// has the highest scheduling priority -- does not spend issue slots spinning.
+#ifndef QC_IDLE_SLEEP
+#define QC_IDLE_SLEEP 1
+#endif
+__device__ __forceinline__ void mbar_wait_idle(uint64_t *bar, uint32_t parity) {
+#if QC_IDLE_SLEEP
+    const uint32_t a = smem_u32(bar);
+    uint64_t t0 = 0;
+    uint32_t it = 0;
+    while (!mbar_try_wait_sleep(a, parity)) {
+        if ((++it & 15u) == 0) {
+            const uint64_t t = globaltimer_ns();
+            if (t0 == 0) t0 = t;
+            else if (t - t0 > 4000000000ull) __trap();
+        }
+    }
+#else
+    mbar_wait(bar, parity);
+#endif
+}
+
 // ---------------------------------------------------------------- programmatic dependent launch
 // The conv kernels are launched with programmatic stream serialization: a kernel may start
 // (prologue, barrier init, TMEM alloc, descriptor prefetch, weight loads) while the previous
@@ -165,6 +188,14 @@ __device__ __forceinline__ void tma_store_2d(const void *map, const void *src, i
     asm volatile(
         "cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(map),
         "r"(smem_u32(src)), "r"(x), "r"(y)
+        : "memory");
+}
+// Non-tensor bulk copy of `bytes` (multiple of 16) contiguous global bytes into shared memory,
+// completing on an mbarrier (one request stream, no per-row addressing).
+__device__ __forceinline__ void bulk_load(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
         : "memory");
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }

@@ -25,6 +25,10 @@
 #include "launch.h"
 #include "prep.cuh"
 
+#ifndef QC_MAX_YSTG
+#define QC_MAX_YSTG 4
+#endif
+
 namespace {
 
 thread_local int g_last_cuda_error = 0;
@@ -680,9 +684,15 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const uint32_t hx = static_cast<uint32_t>(align_up(static_cast<size_t>(nplanes) * plane, 1024));
     const uint32_t hp = is4 ? static_cast<uint32_t>(align_up(static_cast<size_t>(nch) * plane, 1024)) : 0u;
     const uint32_t bres = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * KG8, 1024));
-    const uint32_t ystg = 2u * 128u * static_cast<uint32_t>(tile_row_bytes);   // double-buffered
-    const uint32_t fixed = bres + ystg + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 2048u +
-                           8u * static_cast<uint32_t>(d->r * d->s * nplanes);
+    // output staging ring: 4 buffers when the halo ring keeps >= 3 stages, else 3, else 2
+    int n_ystg = QC_MAX_YSTG;
+    uint32_t ystg = 0, fixed = 0;
+    for (;; --n_ystg) {
+        ystg = static_cast<uint32_t>(n_ystg) * 128u * static_cast<uint32_t>(tile_row_bytes);
+        fixed = bres + ystg + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 2048u +
+                8u * static_cast<uint32_t>(d->r * d->s * nplanes);
+        if (n_ystg == 2 || fixed + 3 * (hx + hp) <= 227u * 1024u) break;
+    }
     if (fixed + 2 * (hx + hp) > 227u * 1024u) return false;
     int stages = static_cast<int>((227u * 1024u - fixed) / (hx + hp));
     stages = std::min(stages, 24);   // deep ring: the halo loads are latency-bound (~6 us each under load)
@@ -709,7 +719,8 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.c_px = g.c_bytes;
     p.halo_flat = ((tap_pair || is4) && (Wh * g.c_bytes) % 8 == 0 && Wh * g.c_bytes / 8 <= 256) ? 1 : 0;
     p.off_ystg = static_cast<uint32_t>(align_up(p.off_hp + hp * stages, 1024));
-    p.ystg_bytes = ystg / 2;
+    p.ystg_bytes = ystg / static_cast<uint32_t>(n_ystg);
+    p.n_ystg = n_ystg;
     p.y_tma = 1;
     p.y_gw = y_gw;
     p.y_gmask = y_gw == 128 ? 7 : (y_gw == 64 ? 3 : 1);
@@ -719,7 +730,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     if (p.n_mma > qc::kHaloMaxMMA) return false;
     p.off_mtab = static_cast<uint32_t>(align_up(p.off_par + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u, 16));
     p.off_bar = static_cast<uint32_t>(align_up(p.off_mtab + 8u * static_cast<uint32_t>(p.n_mma), 8));
-    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 9) * 8 + 16);
+    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 5 + 2 * qc::kMaxYstg + 1) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
     if (pl->smem_bytes > 227u * 1024u) return false;
     p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), act_signed(d), dtype_signed(d->w_t));
@@ -1100,6 +1111,13 @@ qc_status launch_plan(const Exec &ex, Plan &pl, const void *x, const void *w8, c
     p.zx_table = ex.zx ? reinterpret_cast<const int32_t *>(wsb + ex.off_zx) : nullptr;
     p.zw = ex.zw ? ex.d->w_zero : nullptr;
     p.x1 = ex.zw ? reinterpret_cast<const int32_t *>(wsb + ex.off_x1) : nullptr;
+    p.fd_pq = qc::make_fastdiv(static_cast<uint32_t>(p.PQ));
+    p.fd_q = qc::make_fastdiv(static_cast<uint32_t>(p.Q));
+    p.fd_ntn = qc::make_fastdiv(static_cast<uint32_t>(p.n_tiles_n));
+    p.fd_tpr = qc::make_fastdiv(static_cast<uint32_t>(std::max(1, p.S * p.chunks)));
+    p.fd_chunks = qc::make_fastdiv(static_cast<uint32_t>(std::max(1, p.chunks)));
+    p.fd_s = qc::make_fastdiv(static_cast<uint32_t>(std::max(1, p.S)));
+    p.fd_tpi = qc::make_fastdiv(static_cast<uint32_t>(std::max(1, p.tiles_per_img)));
     debug_attach(p, st);
     qc::Launch L;
     L.grid = dim3(static_cast<unsigned>(pl.grid));

@@ -143,7 +143,11 @@ def test_requant_mid_hole_worked_example():
 @pytest.mark.parametrize("family", list(FAMILY_SHAPES))
 @pytest.mark.parametrize("bits", [8, 4])
 def test_tflite_rounding_every_kernel(family, bits):
+    """TFLite rounding on every kernel that takes it (the channel-major kernel does not: its
+    epilogue would spill registers; its 1x1 layers then run on the im2col kernel)."""
     cs, kern, bn = FAMILY_SHAPES[family]
+    if family == "channel":
+        kern, bn = None, 0
     li = make_layer_inputs(cs, bits, seed=5 + bits, relu=False, signed_out=True)
     rng = np.random.default_rng(7 + bits)
     m, n = _requant_domain(cs.k, rng)
