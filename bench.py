@@ -464,12 +464,25 @@ def run_trunk(args):
     else:                                              # C5: 256 images over all GPUs
         per_gpu = shard_bounds(rank, world, args.global_batch)[1]
         global_batch, scaling = args.global_batch, "strong"
+    from paper_conf_icpp_hanhyylhgwwlq20_b200 import tuning
+    plans_path = args.plans if args.plans not in ("", "none") else None
+    if args.plans == "":
+        auto = os.path.join(ROOT, "plans", f"resnet50_trunk_a{args.bits}_b{per_gpu}.json")
+        plans_path = auto if os.path.exists(auto) else None
+    n_plans = tuning.load_plans(plans_path) if plans_path else 0
     trunk = Trunk(args.bits, per_gpu, device, dist_ctx, rank=rank)
+    plans_note = (f"profile-run table {os.path.relpath(plans_path, ROOT)} ({n_plans} shapes)"
+                  if n_plans else "default rule")
     if args.tune:
+        entries = tuning.tune_layers(trunk.layers[1:], iters=5)     # the stem runs in s2d form
         for L in trunk.layers:
-            trunk.qc.qconv_autotune(L["desc"], L["x"], L["w"], L["bias"], L["m"], L["n"],
-                                    y=L["y"], iters=5)
             L["plan"] = trunk.qc.qconv_debug_plan(L["desc"])
+        plans_note = "autotuned in this run"
+        if args.save_plans and rank == 0:
+            os.makedirs(os.path.dirname(os.path.abspath(args.save_plans)), exist_ok=True)
+            tuning.save_plans(args.save_plans, entries,
+                              {"workload": f"resnet50_trunk_a{args.bits}", "per_gpu_batch": per_gpu,
+                               "how": "qconv_autotune, 5 timed launches per candidate, CUDA events"})
 
     if args.profile_steps:
         for _ in range(args.warmup + args.profile_steps):
@@ -613,7 +626,7 @@ def run_trunk(args):
                        "l2": "inputs > L2: 154 MB fp32 stem input and ~2.4 GB of trunk traffic per step "
                              "(at 256 images per GPU)",
                        "graph": "one CUDA graph per step (PDL between the conv kernels), replayed",
-                       "plans": "autotuned" if args.tune else "default rule"},
+                       "plans": plans_note},
             "tops": trunk.ops_per_step / (ms_per_step / 1e3) / 1e12,
             "roofline": {"bound": "tensor", "kernel": "the 53 conv launches (qconv_halo / qconv_t / qconv_fwd / qconv_fwd2 kernels)",
                          "achieved": achieved_tops, "peak": peaks["int8_tops"],
@@ -749,7 +762,7 @@ def run_layers(args):
     peaks = load_peaks()
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=device)
     shapes = workload_layers(args.workload, bits)
-    results, bad = [], []
+    results, bad, tuned = [], [], []
     total_ops = total_us = total_roof = 0.0
     clk = ClockSampler(0)
     clk.start()
@@ -774,7 +787,10 @@ def run_layers(args):
             x = W.device_post_relu_codes((cs.n, cs.h, cs.w, c_st), bits, W.layer_seed(200 + i), device)
         y = qc.qconv2d_forward(d, x, w, b, mm, nn)
         if args.tune:
-            qc.qconv_autotune(d, x, w, b, mm, nn, y=y, iters=5)
+            best, tus = qc.qconv_autotune(d, x, w, b, mm, nn, y=y, iters=5)
+            from paper_conf_icpp_hanhyylhgwwlq20_b200 import tuning
+            tuned.append({"name": cs.name, "desc": tuning.desc_fields(d), "kernel": best["kernel"],
+                          "kernel_name": best["kernel_name"], "bn": best["bn"], "us": tus})
         plan = qc.qconv_debug_plan(d)
 
         def launch():
@@ -844,6 +860,9 @@ def run_layers(args):
     if args.layers_json:
         with open(args.layers_json, "w") as f:
             json.dump(line, f, indent=1)
+    if args.save_plans and tuned:
+        from paper_conf_icpp_hanhyylhgwwlq20_b200 import tuning
+        tuning.save_plans(args.save_plans, tuned, {"workload": args.workload, "bits": bits})
     return 0
 
 
@@ -860,6 +879,9 @@ def main():
     ap.add_argument("--batch", type=int, default=0, help="weak scaling: images per GPU")
     ap.add_argument("--impl", default="ours", choices=("ours", "reference"))
     ap.add_argument("--tune", action="store_true", help="profile-run tile search before timing")
+    ap.add_argument("--plans", default="", help="tile-search table to apply ('' = plans/<workload>.json "
+                                                "if present, 'none' = the default rule)")
+    ap.add_argument("--save-plans", default="", help="write the --tune results to this table")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-verify", action="store_true")
