@@ -157,13 +157,12 @@ class Trunk:
         self.x_float = torch.relu(torch.randn((batch, stem.h, stem.w, stem.c), generator=g,
                                               device=device, dtype=torch.float32))
         self.s_in = stem_scale(bits)
-        # the stem (7x7/s2, C=3) runs in space-to-depth form: 4x4/s1 over C=16 byte codes,
-        # written directly by the fused fp32 quantize (qconv_quantize_pack_s2d)
+        # the stem (7x7/s2, C=3) takes the fp32 image: qconv2d_forward_quantize runs it as one
+        # kernel (the fp32 rows are quantized inside it, straight into its space-to-depth
+        # operand tile: 4x4/s1 over 16 byte-coded channels)
         self.stem_desc = qc.make_desc(batch, stem.h, stem.w, stem.c, stem.k, stem.r, stem.s,
                                       stride=stem.stride, pad=stem.pad, x_t=x_t, w_t=W.S8,
                                       y_t=x_t, relu=True)
-        d2 = qc.qconv_s2d_desc(self.stem_desc)
-        self.x_q = torch.empty((d2.n, d2.h, d2.w, d2.c), dtype=torch.uint8, device=device)
         # res2 input: max-pool is outside the method -> separately drawn codes
         rng = np.random.default_rng(W.SEED_BASE + 31 * rank + 1)
         codes = W.post_relu_codes_fast(rng, (batch, 56, 56, 64), bits)
@@ -177,8 +176,9 @@ class Trunk:
         block_in = None
         for (cs, c_st, i), (wb, pb) in zip(specs, params):
             if i == 0:
-                w_prep = qc.qconv_prepare_weights_s2d(self.stem_desc, wb)
-                d = qc.qconv_s2d_desc(self.stem_desc)
+                d = qc.qconv_desc.from_buffer_copy(self.stem_desc)
+                w_prep = qc.qconv_prepare_weights(d, wb)
+                d.w_prepared = 1
             else:
                 d = qc.make_desc(cs.n, cs.h, cs.w, c_st, cs.k, cs.r, cs.s, stride=cs.stride,
                                  pad=cs.pad, x_t=x_t, w_t=w_t, y_t=x_t, relu=True)
@@ -188,7 +188,7 @@ class Trunk:
             y = torch.empty((cs.n, p, q, cs.k * bits // 8), dtype=torch.uint8, device=device)
             role = W.RESNET50_LAYERS[i]["role"]
             if role == "stem":
-                src = self.x_q
+                src = self.x_float
             elif role == "2a":
                 block_in = self.res2_in if cs.name.startswith("res2a") else cur
                 src = block_in
@@ -198,9 +198,11 @@ class Trunk:
                 src = cur
             assert src.shape[1] == d.h and src.shape[2] == d.w, cs.name
             ops, nbytes = layer_algorithmic(cs, bits)
+            if i == 0:                      # the stem reads the fp32 image, not codes
+                nbytes += cs.n * cs.h * cs.w * cs.c * (4 - bits / 8)
+            plan = qc.qconv_debug_plan_quantize(d) if i == 0 else qc.qconv_debug_plan(d)
             self.layers.append(dict(name=cs.name, shape=cs, desc=d, w=w_prep, bias=pb[0], m=pb[1],
-                                    n=pb[2], x=src, y=y, ops=ops, bytes=nbytes,
-                                    plan=qc.qconv_debug_plan(d)))
+                                    n=pb[2], x=src, y=y, ops=ops, bytes=nbytes, plan=plan))
             if role in ("stem", "2a", "2b", "2c"):
                 cur = y
         self.out = cur
@@ -210,33 +212,25 @@ class Trunk:
     def ops_per_step(self):
         return sum(L["ops"] for L in self.layers)
 
-    @property
-    def quantize_bytes(self):
-        """Algorithmic bytes of the stem quantization: the fp32 input read + its codes written
-        packed at the layer's bit width (the space-to-depth byte layout is an implementation
-        choice, not algorithmic traffic)."""
-        d = self.stem_desc
-        return d.n * d.h * d.w * d.c * 4 + d.n * d.h * d.w * d.c * self.bits // 8
-
     def launches_per_step(self):
-        return 1 + len(self.layers)
+        return len(self.layers)
 
     def step(self, events=None, x_float=None, before_last=None):
         """Enqueue one step on the current stream; events[i] recorded after launch i;
         before_last() runs just before the last layer is enqueued (e2e: the wait for the D2H
         of the previous step's output, which that layer overwrites)."""
         qc = self.qc
-        qc.qconv_quantize_pack_s2d(self.stem_desc, self.x_float if x_float is None else x_float,
-                                   self.s_in, out=self.x_q)
-        if events is not None:
-            events[0].record()
         last = len(self.layers) - 1
         for j, L in enumerate(self.layers):
             if j == last and before_last is not None:
                 before_last()
-            qc.qconv2d_forward(L["desc"], L["x"], L["w"], L["bias"], L["m"], L["n"], y=L["y"])
+            if j == 0:                  # fused fp32 quantize + stem
+                qc.qconv2d_forward_quantize(L["desc"], self.x_float if x_float is None else x_float,
+                                            self.s_in, L["w"], L["bias"], L["m"], L["n"], y=L["y"])
+            else:
+                qc.qconv2d_forward(L["desc"], L["x"], L["w"], L["bias"], L["m"], L["n"], y=L["y"])
             if events is not None:
-                events[j + 1].record()
+                events[j].record()
 
 
 # ----------------------------------------------------------------------------- clocks
@@ -475,7 +469,7 @@ def run_trunk(args):
                   if n_plans else "default rule")
     if args.tune:
         entries = tuning.tune_layers(trunk.layers[1:], iters=5)     # the stem runs in s2d form
-        for L in trunk.layers:
+        for L in trunk.layers[1:]:
             L["plan"] = trunk.qc.qconv_debug_plan(L["desc"])
         plans_note = "autotuned in this run"
         if args.save_plans and rank == 0:
@@ -493,7 +487,7 @@ def run_trunk(args):
     stream = torch.cuda.Stream(device=device)
     nL = trunk.launches_per_step()
     # (1) the timed region: one CUDA graph of the whole step with nothing inside but the
-    #     54 launches (the conv kernels use programmatic dependent launch, so a kernel's
+    #     53 launches (the conv kernels use programmatic dependent launch, so a kernel's
     #     prologue overlaps the previous kernel's tail -- timing events between launches
     #     would serialize that), replayed K times
     # (2) a second pass, right after, of K graphs with a timing event after every launch:
@@ -561,8 +555,7 @@ def run_trunk(args):
     value = global_batch / (ms_per_step / 1000.0)
 
     peaks = load_peaks()
-    conv_ms = per_launch[:, 1:].mean(axis=0)           # per conv layer, averaged over steps
-    q_ms = per_launch[:, 0].mean()
+    conv_ms = per_launch.mean(axis=0)                  # per conv layer, averaged over steps
     conv_ops = np.array([L["ops"] for L in trunk.layers], dtype=np.float64)
     conv_bytes = np.array([L["bytes"] for L in trunk.layers], dtype=np.float64)
     conv_total_ms = float(conv_ms.sum())
@@ -611,9 +604,8 @@ def run_trunk(args):
                            "frac_hbm": L["bytes"] / t_s / 1e9 / peaks["hbm_gbs"]})
         if args.layers_json:
             with open(args.layers_json, "w") as f:
-                json.dump({"layers": layers, "quantize_us": q_ms * 1e3, "families": families,
+                json.dump({"layers": layers, "families": families,
                            "ms_per_step": ms_per_step}, f, indent=1)
-        qgbs = trunk.quantize_bytes / (q_ms / 1e3) / 1e9
         line = {
             "metric": METRIC, "value": value, "unit": "images/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
@@ -648,9 +640,10 @@ def run_trunk(args):
                          "instrumented_ms_per_step": instr_ms_per_step,
                          "algorithmic_ops_per_step": float(conv_ops.sum()),
                          "algorithmic_bytes_per_step": float(conv_bytes.sum())},
-            "quantize_pack": {"kernel": "quantize_s2d_kernel (fp32 -> space-to-depth codes)",
-                              "us": q_ms * 1e3, "gbs": qgbs, "frac_hbm": qgbs / peaks["hbm_gbs"],
-                              "algorithmic_bytes": trunk.quantize_bytes},
+            "quantize_pack": {"kernel": "fused into the stem (qconv2d_forward_quantize: the halo kernel's "
+                                        "converter warps quantize the TMA-loaded fp32 rows)",
+                              "stem_us": conv_ms[0] * 1e3,
+                              "stem_algorithmic_bytes": float(conv_bytes[0])},
             "parity": parity,
             "e2e": e2e, "cpu_baseline": cpu, "clocks": clocks,
             "gpu_launches": args.steps * nL,   # our kernels in the timed region

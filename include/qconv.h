@@ -208,6 +208,27 @@ qc_status qconv2d_forward_dequant(const qconv_desc *d, const void *x, const void
                                   void *workspace, size_t ws_bytes, void *stream);
 
 /*
+ * qconv2d_forward_quantize -- the quantization step fused with the convolution (P:L257,
+ * P:L263): float activations in, y = qconv2d_forward(d, q(x), ...) out, where q quantizes
+ * every element with reading Z4 (one fp32 multiply by fl32(1/in_scale), round to nearest even,
+ * + d->x_zero, clamp to the d->x_t code range; NaN -> x_zero).
+ *   x         device, fp32 or bf16 (xt) NHWC [n, h, w, c] with the true channel count
+ *   in_scale  > 0 and finite
+ *   other arguments as qconv2d_forward; workspace >= qconv2d_quantize_workspace_size(d, xt)
+ * The image stem (stride 2, dilation 1, 4*c <= 16, fp32, x_zero = 0, no w_zero, w*c % 4 == 0,
+ * w*c <= 1024: the ResNet / VGG C = 3 stem) runs as ONE kernel: the TMA loads the fp32 rows and
+ * the kernel's converter warps quantize them straight into its space-to-depth operand tile
+ * (no code tensor in global memory).  Any other descriptor quantizes into the workspace and
+ * then runs qconv2d_forward (two launches, same bytes).
+ * Errors: as qconv2d_forward; UNSUPPORTED also for 4-bit x_t with odd c outside the fused case.
+ */
+size_t qconv2d_quantize_workspace_size(const qconv_desc *d, qc_ftype xt);
+qc_status qconv2d_forward_quantize(const qconv_desc *d, const void *x, qc_ftype xt, float in_scale,
+                                   const void *w, const int32_t *bias, const int32_t *multiplier,
+                                   const int32_t *shift, void *y, void *workspace, size_t ws_bytes,
+                                   void *stream);
+
+/*
  * Launch plans and the per-shape tile search (the paper's "auto-search ... choose the
  * best ones through profile runs", section 5.1).
  *   kernel : QC_KERNEL_IM2COL   im2col implicit GEMM, one CTA per 128-pixel tile
@@ -244,6 +265,8 @@ typedef struct {
 } qconv_plan;
 
 qc_status qconv_debug_plan(const qconv_desc *d, qconv_plan *out);
+/* The plan qconv2d_forward_quantize launches (prologue bit 16: a separate quantize launch). */
+qc_status qconv_debug_plan_quantize(const qconv_desc *d, qc_ftype xt, qconv_plan *out);
 qc_status qconv_plan_set(const qconv_desc *d, const qconv_plan *choice);
 void qconv_plan_clear(void);
 int32_t qconv_plan_candidates(const qconv_desc *d, qconv_plan *out, int32_t cap);

@@ -92,9 +92,15 @@ def _lib():
         L.qconv2d_forward.restype = i32
         L.qconv2d_forward_dequant.argtypes = [dp, vp, vp, vp, vp, vp, vp, sz, vp]
         L.qconv2d_forward_dequant.restype = i32
+        L.qconv2d_quantize_workspace_size.argtypes = [dp, i32]
+        L.qconv2d_quantize_workspace_size.restype = sz
+        L.qconv2d_forward_quantize.argtypes = [dp, vp, i32, f32, vp, vp, vp, vp, vp, vp, sz, vp]
+        L.qconv2d_forward_quantize.restype = i32
         pp = ctypes.POINTER(qconv_plan)
         L.qconv_debug_plan.argtypes = [dp, pp]
         L.qconv_debug_plan.restype = i32
+        L.qconv_debug_plan_quantize.argtypes = [dp, i32, pp]
+        L.qconv_debug_plan_quantize.restype = i32
         L.qconv_plan_set.argtypes = [dp, pp]
         L.qconv_plan_set.restype = i32
         L.qconv_plan_clear.argtypes = []
@@ -269,10 +275,37 @@ def qconv2d_forward_dequant(d: qconv_desc, x, w, bias=None, scale=None, y=None, 
     return y
 
 
+def qconv2d_forward_quantize(d: qconv_desc, x, in_scale: float, w, bias=None, multiplier=None,
+                             shift=None, y=None, workspace=None, stream=None):
+    """Float activations in: quantize (Z4, d.x_zero, d.x_t range) fused with the convolution
+    (include/qconv.h); the C = 3 image stem runs as one kernel."""
+    import torch
+    assert x.is_cuda and x.is_contiguous() and x.dtype in (torch.float32, torch.bfloat16)
+    xt = QC_BF16 if x.dtype == torch.bfloat16 else QC_F32
+    if y is None:
+        y = _out_tensor(d, x.device)
+    need = int(_lib().qconv2d_quantize_workspace_size(ctypes.byref(d), xt))
+    if need and workspace is None:
+        workspace = torch.empty(need, dtype=torch.uint8, device=x.device)
+    ws_bytes = 0 if workspace is None else workspace.numel() * workspace.element_size()
+    _check("qconv2d_forward_quantize", _lib().qconv2d_forward_quantize(
+        ctypes.byref(d), _ptr(x), xt, float(in_scale), _ptr(w), _ptr(bias), _ptr(multiplier),
+        _ptr(shift), _ptr(y), _ptr(workspace), ws_bytes, _stream(stream)))
+    return y
+
+
 def qconv_debug_plan(d: qconv_desc) -> dict:
     """The launch plan qconv2d_forward would use for `d` (kernel family, tiles, grid, ...)."""
     p = qconv_plan()
     _check("qconv_debug_plan", _lib().qconv_debug_plan(ctypes.byref(d), ctypes.byref(p)))
+    return p.as_dict()
+
+
+def qconv_debug_plan_quantize(d: qconv_desc, xt: int = QC_F32) -> dict:
+    """The launch plan of qconv2d_forward_quantize for `d` (float activations of type xt)."""
+    p = qconv_plan()
+    _check("qconv_debug_plan_quantize", _lib().qconv_debug_plan_quantize(ctypes.byref(d), int(xt),
+                                                                         ctypes.byref(p)))
     return p.as_dict()
 
 
@@ -393,7 +426,7 @@ class QConv2d:
 
 
 __all__ = ["qconv_quantize_pack", "qconv_requant_params", "qconv_prepare_weights",
-           "qconv2d_forward_dequant", "qconv_debug_plan", "qconv_plan_candidates",
+           "qconv2d_forward_dequant", "qconv2d_forward_quantize", "qconv_debug_plan", "qconv_debug_plan_quantize", "qconv_plan_candidates",
            "qconv_plan_set", "qconv_plan_clear", "qconv_autotune", "qconv_plan",
            "QC_F32_OUT", "QC_BF16_OUT", "QC_ROUND_SINGLE", "QC_ROUND_TFLITE",
            "QC_KERNEL_AUTO", "QC_KERNEL_IM2COL", "QC_KERNEL_PAIR", "QC_KERNEL_HALO",

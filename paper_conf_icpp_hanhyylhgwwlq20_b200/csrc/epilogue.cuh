@@ -79,6 +79,11 @@ struct ConvParams {
     uint32_t ystg_bytes;              // one staging buffer
     int32_t n_ystg;                   // halo / channel-major: staging buffers in the ring (2..4)
     int32_t n_wide;                   // channel-major 4-bit: widened operand slots (2..4)
+    // halo kernel with fused fp32 quantization of the space-to-depth stem (F32 instantiation):
+    // quantize_one parameters and the original image geometry
+    float q_inv_s, q_flo, q_fhi;
+    int32_t q_z, q_qmin, q_qmax;
+    int32_t f_w, f_c, f_pad_h, f_pad_w, f_rowbytes;
     int32_t b_res;                    // channel-major: the CTA's weights resident at off_bres
     const uint8_t *x_lin;             // channel-major 4-bit, 1x1/s1/p0, one K chunk: activations read
                                       // as one contiguous bulk copy per tile (else null: im2col TMA)

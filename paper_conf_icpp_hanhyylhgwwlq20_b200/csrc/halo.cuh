@@ -18,12 +18,97 @@
 // have no counterpart: the hardware gathers, shared memory reuses.
 #pragma once
 #include "epilogue.cuh"
+#include "quant.cuh"
 
 namespace qc {
 
 
-template <bool IS4, int OUT>
-__global__ void __launch_bounds__(IS4 ? 512 : 384, 1)
+// Fused fp32 quantization of the space-to-depth stem (F32): the producer TMA-loads the tile's
+// 2*HR fp32 input rows (a 4-D [n][h][w*c/4][4] view: rows outside the image are zero-filled, and
+// quantize to the zero point, the space-to-depth padding code), and the converter warps quantize
+// them (reading Z4: one fp32 multiply by fl32(1/scale), round to nearest even, + z, clamp; NaN ->
+// z) straight into the byte-coded halo X2[i][j][(2b+b')*c + cc] = q(x[2i+b-pad_h, 2j+b'-pad_w, cc])
+// -- no X2 tensor in global memory and no separate quantize launch.
+// NaN-propagating float min / max (fminf / fmaxf return the other operand for a NaN).
+__device__ __forceinline__ float fmax_nan(float a, float b) {
+    float r;
+    asm("max.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b));
+    return r;
+}
+__device__ __forceinline__ float fmin_nan(float a, float b) {
+    float r;
+    asm("min.NaN.f32 %0, %1, %2;" : "=f"(r) : "f"(a), "f"(b));
+    return r;
+}
+
+// quantize_one (quant.cuh, reading Z4) without branches: the clamp to the integer bounds
+// [qmin - z, qmax - z] in the float domain commutes with round-to-nearest-even, so no integer
+// clamp follows, and a NaN passes the NaN-propagating clamp and converts to 0, i.e. code z.
+__device__ __forceinline__ int32_t f32_q(const ConvParams &p, float x) {
+    const float t = fmin_nan(fmax_nan(__fmul_rn(x, p.q_inv_s), p.q_flo), p.q_fhi);
+    return __float2int_rn(t) + p.q_z;
+}
+
+// One space-to-depth pixel X2[i][j] (16 code bytes, channel (2b+b')*C + cc; the 4C..15 tail
+// holds the zero point) from the two staged fp32 input rows 2i - pad_h, +1.  addr[blk] is the
+// address of input pixel (2i + (blk >> 1) - pad_h, 2j + (blk & 1) - pad_w), or of a zeroed
+// 16-byte area when that pixel is outside the image (+0.0 quantizes to the zero point).
+template <int C>
+__device__ __forceinline__ void f32_s2d_pixel(const ConvParams &p, const uint32_t (&addr)[4], uint32_t (&w)[4]) {
+    int32_t code[16];
+#pragma unroll
+    for (int blk = 0; blk < 4; ++blk) {
+#pragma unroll
+        for (int cc = 0; cc < C; ++cc) {
+            float v;
+            asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr[blk] + 4u * cc));
+            code[blk * C + cc] = f32_q(p, v);
+        }
+    }
+#pragma unroll
+    for (int k = 4 * C; k < 16; ++k) code[k] = p.q_z;
+    // codes are in [qmin, qmax] already: the saturating packs only place the bytes
+    if (p.q_qmin < 0) {
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+            w[k] = pack_sat_s8(code[4 * k + 1], code[4 * k], pack_sat_s8(code[4 * k + 3], code[4 * k + 2], 0u));
+    } else {
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+            w[k] = pack_sat_u8(code[4 * k + 1], code[4 * k], pack_sat_u8(code[4 * k + 3], code[4 * k + 2], 0u));
+    }
+}
+
+// Per-thread source layout of X2 column j: byte offsets within a staged row pair of its four
+// input pixels and a mask of those inside the image.
+__device__ __forceinline__ uint32_t f32_s2d_offsets(const ConvParams &p, int j, uint32_t (&off)[4]) {
+    uint32_t ok = 0;
+#pragma unroll
+    for (int blk = 0; blk < 4; ++blk) {
+        const int ww = 2 * j + (blk & 1) - p.f_pad_w;
+        const bool in = ww >= 0 && ww < p.f_w;
+        off[blk] = (blk >> 1) * static_cast<uint32_t>(p.f_rowbytes) + 4u * static_cast<uint32_t>((in ? ww : 0) * p.f_c);
+        ok |= in ? (1u << blk) : 0u;
+    }
+    return ok;
+}
+__device__ __forceinline__ void f32_s2d_addr(uint32_t rows, const uint32_t (&off)[4], uint32_t ok, uint32_t zero,
+                                             uint32_t (&addr)[4]) {
+#pragma unroll
+    for (int blk = 0; blk < 4; ++blk) addr[blk] = (ok >> blk) & 1u ? rows + off[blk] : zero;
+}
+
+// Position in an NS-stage mbarrier ring (stage, phase parity), advanced without divisions.
+struct RingPos {
+    int stage = 0;
+    uint32_t phase = 0;
+    __device__ __forceinline__ void next(int ns) {
+        if (++stage == ns) { stage = 0; phase ^= 1u; }
+    }
+};
+
+template <bool IS4, int OUT, bool F32 = false>
+__global__ void __launch_bounds__((IS4 || F32) ? 512 : 384, 1)
 qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap bmap,
                   const __grid_constant__ CUtensorMap ymap, const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -53,7 +138,8 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
     // is on the kernel's critical path, so it must not wait behind epilogue instructions.
     constexpr int kEpi0 = 0;
     constexpr int kCvt0 = kNumEpiWarps;
-    constexpr int kCtl0 = kNumEpiWarps + (IS4 ? kNumCvtWarps : 0);
+    constexpr bool kCvt = IS4 || F32;                // converter warps present
+    constexpr int kCtl0 = kNumEpiWarps + (kCvt ? kNumCvtWarps : 0);
     constexpr int kProd = kCtl0, kStorer = kCtl0 + 1, kMma = kCtl0 + 3;
     griddep_launch_dependents();
     if (warp == kProd && lane == 0) {
@@ -81,6 +167,16 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
+    // Tiles of this CTA: round robin over the grid, or -- for the fused fp32 stem -- one
+    // contiguous run of output rows, so a tile's space-to-depth halo shares HR-1 of its HR rows
+    // with the previous tile's (converted once, copied forward) and only two new fp32 rows are
+    // loaded per tile.  (F32 always has one N tile: K <= 256.)
+    int t_first = static_cast<int>(blockIdx.x), t_step = static_cast<int>(gridDim.x), t_end = p.num_tiles;
+    if (F32) {
+        t_first = static_cast<int>(static_cast<int64_t>(blockIdx.x) * p.num_tiles / gridDim.x);
+        t_end = static_cast<int>(static_cast<int64_t>(blockIdx.x + 1) * p.num_tiles / gridDim.x);
+        t_step = 1;
+    }
     // all tiles of this CTA share one N tile (grid is a multiple of n_tiles_n)
     const int n0 = (static_cast<int>(blockIdx.x) % p.n_tiles_n) * p.BN;
 
@@ -88,12 +184,13 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         // ===================== output storer (see trans.cuh) =====================
         if (lane == 0) {
             int it = 0;
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
-                const int b = it % NB;
+            int b = 0, bprev = 0;                   // staging buffer of this / the previous tile
+            uint32_t bphase = 0;
+            for (int tile = t_first; tile < t_end; tile += t_step, ++it) {
                 const int mt = p.fd_ntn.div(tile);
                 const int img = p.fd_tpi.div(mt);
                 const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
-                mbar_wait(&sfull[b], static_cast<uint32_t>(it / NB) & 1u);
+                mbar_wait(&sfull[b], bphase);
                 {
                     constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
                     for (int gi = 0; gi < p.n_ygroups; ++gi)
@@ -103,7 +200,9 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 bulk_commit();
                 // keep two stores in flight: the previous one has read its buffer -> release it
                 bulk_wait_read<1>();
-                if (it > 0) mbar_arrive(&sfree[(it - 1) % NB]);
+                if (it > 0) mbar_arrive(&sfree[bprev]);
+                bprev = b;
+                if (++b == NB) { b = 0; bphase ^= 1u; }
                 trace_ev(p, 7, it);
             }
             bulk_wait<0>();
@@ -118,20 +217,30 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             if (leader) mbar_arrive_expect_tx(bfull, p.b_res_bytes);
             if (leader) tma_load_3d(smem + p.off_bres, &bmap, bfull, 0, n0, 0);
             int g = 0;
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
+            RingPos rp;
+            for (int tile = t_first; tile < t_end; tile += t_step, ++g, rp.next(NS)) {
                 const int mt = p.fd_ntn.div(tile);
                 const int img = p.fd_tpi.div(mt);
                 const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
-                const int stage = g % NS;
-                const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
-                mbar_wait(&hempty[stage], phase ^ 1u);
+                const int stage = rp.stage;
+                mbar_wait(&hempty[stage], rp.phase ^ 1u);
                 if (leader) trace_ev(p, 0, g);
-                if (leader) mbar_arrive_expect_tx(&hfull[stage], p.halo_tx);
-                uint8_t *dst = IS4 ? smem + p.off_hp + stage * p.hp_stage_bytes
-                                   : smem + p.off_hx + stage * p.hx_stage_bytes;
-                if (p.halo_flat) {     // rows of Wh pixels as int64 elements: few long TMA rows
+                uint8_t *dst = kCvt ? smem + p.off_hp + stage * p.hp_stage_bytes
+                                    : smem + p.off_hx + stage * p.hx_stage_bytes;
+                if (F32) {
+                    // fp32 input row pairs (2*(p0+hr) - pad_h, +1) of the original image; a
+                    // continuation tile only needs the pair of its last halo row
+                    const bool cont = tile != t_first && p0 != 0 && p.Rt < p.HR;
+                    const int hr0 = cont ? p.HR - p.Rt : 0;
+                    if (leader) mbar_arrive_expect_tx(&hfull[stage], static_cast<uint32_t>(2 * (p.HR - hr0) * p.f_rowbytes));
+                    for (int hr = hr0; hr < p.HR; ++hr)
+                        tma_load_4d(dst + 2 * (hr - hr0) * p.f_rowbytes, &hmap, &hfull[stage], 0, 0,
+                                    2 * (p0 + hr) - p.f_pad_h, img);
+                } else if (p.halo_flat) {
+                    if (leader) mbar_arrive_expect_tx(&hfull[stage], p.halo_tx);     // rows of Wh pixels as int64 elements: few long TMA rows
                     if (leader) tma_load_3d(dst, &hmap, &hfull[stage], -p.pad_w * (p.c_px / 8), p0 - p.pad_h, img);
                 } else {
+                    if (leader) mbar_arrive_expect_tx(&hfull[stage], p.halo_tx);
                     if (leader) tma_load_5d(dst, &hmap, &hfull[stage], 0, -p.pad_w, p0 - p.pad_h, img, 0);
                 }
             }
@@ -171,27 +280,39 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             int it = 0;
             int stage = 0;                           // ring position, advanced incrementally
             uint32_t phase = 0;
-            for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+            int f_base = 0;                          // F32: ring row of the tile's halo row 0
+            for (int tile = t_first; tile < t_end; tile += t_step, ++it) {
                 const int buf = it & 1;
                 const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
                 mbar_wait(&tempty[buf], acc_phase ^ 1u);
                 if (leader) trace_ev(p, 2, it);
-                mbar_wait(IS4 ? &hready[stage] : &hfull[stage], phase);
+                mbar_wait(kCvt ? &hready[stage] : &hfull[stage], phase);
                 if (leader) trace_ev(p, 3, it);
                 __syncwarp();
                 tc_fence_after();
                 if (leader) trace_ev(p, 1, it);
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
-                const uint32_t alo0 = static_cast<uint32_t>(adesc_st) +
-                                      ((static_cast<uint32_t>(stage) * p.hx_stage_bytes) >> 4);
-                // fully unrolled over the precomputed per-MMA offsets (registers).  Measured: the
-                // tensor pipe takes one of these M128 x N64 x K32 MMAs per ~120-150 cycles (grouping
-                // four under one election, or interleaving four tiles' accumulators, changed nothing)
-#pragma unroll
-                for (int i = 0; i < kHaloMaxMMA; ++i) {
-                    if (i < nmma)
-                        mma_i8_warp_lo(d_tmem, alo0 + aoff[i], ahi, blo0 + boff[i], bhi, p.idesc, i > 0 ? 1u : 0u);
+                uint32_t alo0 = static_cast<uint32_t>(adesc_st) +
+                                ((static_cast<uint32_t>(stage) * p.hx_stage_bytes) >> 4);
+                if (F32) {   // the tile's window of the converter's code-row ring (same sequence)
+                    const int mt = p.fd_ntn.div(tile);
+                    const int p0 = (mt - p.fd_tpi.div(mt) * p.tiles_per_img) * p.Rt;
+                    if (tile != t_first && p0 != 0 && p.Rt < p.HR) {
+                        f_base += p.Rt;
+                        if (f_base >= p.HR + p.Rt) f_base -= p.HR + p.Rt;
+                    } else {
+                        f_base = 0;
+                    }
+                    alo0 = static_cast<uint32_t>(adesc_st) + ((static_cast<uint32_t>(f_base) * static_cast<uint32_t>(p.Wh)));
                 }
+                // fully unrolled and branch-free over the precomputed per-MMA offsets (MMAs past
+                // n_mma are predicated off).  The tensor pipe takes an M128 x N64 x K32 MMA from
+                // shared memory per 52 cycles (scripts/micro/mma_bench3.cu); guarded by a branch
+                // each, the issue chain paced them at ~150-270.
+#pragma unroll
+                for (int i = 0; i < kHaloMaxMMA; ++i)
+                    mma_i8_warp_lo_if(d_tmem, alo0 + aoff[i], ahi, blo0 + boff[i], bhi, p.idesc, i > 0 ? 1u : 0u,
+                                      i < nmma ? 1u : 0u);
                 if (leader) trace_ev(p, 11, it);
                 mma_commit_warp(&hempty[stage]);
                 if (leader) trace_ev(p, 12, it);
@@ -215,24 +336,26 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         const int nchunks = p.BN / 32;
         const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
         fill_epilogue_params<OUT>(p, par, chunk_info, n0, ew, lane, false);
+        const uint32_t cinfo_base = smem_u32(chunk_info);
+        const uint32_t taddr0 = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16);
         int it = 0;
-        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+        int sb = 0;                                      // staging buffer, advanced incrementally
+        uint32_t sphase = 0;
+        for (int tile = t_first; tile < t_end; tile += t_step, ++it) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
             mbar_wait(&tfull[buf], acc_phase);
             if (ew == 0 && lane == 0) trace_ev(p, 5, it);
             tc_fence_after();
-            const uint32_t taddr = tmem_base + (static_cast<uint32_t>(quarter * 32) << 16) +
-                                   static_cast<uint32_t>(buf * p.BN);
-            const int sb = it % NB;
-            mbar_wait(&sfree[sb], (static_cast<uint32_t>(it / NB) & 1u) ^ 1u);
+            const uint32_t taddr = taddr0 + static_cast<uint32_t>(buf * p.BN);
+            mbar_wait(&sfree[sb], sphase ^ 1u);
             const uint32_t ystg_it = ystg_base + static_cast<uint32_t>(sb) * p.ystg_bytes;
             // TMEM loads double-buffered: chunk ci+2 is in flight while chunk ci is requantized
             uint32_t va[32], vb[32];
             auto process = [&](uint32_t (&v)[32], int ci) {
                 const int col0 = ci * 32;
                 const uint32_t pa = par_base + 16u * col0;
-                const int4 cinfo = chunk_info[ci];
+                const int4 cinfo = lds128(cinfo_base + 16u * static_cast<uint32_t>(ci));
                 epi_requant16<OUT, false, 0>(p, v, pa, cinfo, n0 + col0, 0, 0, 0, 0);
                 epi_requant16<OUT, false, 16>(p, v, pa, cinfo, n0 + col0, 0, 0, 0, 0);
                 if (row_ok) {
@@ -240,7 +363,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                     stage16<OUT, 16>(p, v, ystg_it, srow, col0 + 16);
                 }
             };
-            if (!IS4) {   // 8-bit kernels (384 threads) have the registers to double-buffer
+            if (!kCvt) {  // 384-thread kernels have the registers to double-buffer
                 __syncwarp();
                 if (half < nchunks) tmem_ld_32x32b_x32(taddr + half * 32, va);
                 for (int ci = half; ci < nchunks; ci += 4) {
@@ -255,12 +378,15 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                     process(vb, ci + 2);
                 }
             } else {
+                if (ew == 0 && lane == 0) trace_ev(p, 10, it);
                 for (int ci = half; ci < nchunks; ci += 2) {
                     __syncwarp();
                     tmem_ld_32x32b_x32(taddr + ci * 32, va);
                     tmem_wait_ld();
+                    if (ew == 0 && lane == 0) trace_ev(p, 13, it);
                     process(va, ci);
                 }
+                if (ew == 0 && lane == 0) trace_ev(p, 14, it);
             }
             tc_fence_before();
             fence_proxy_async_smem();                 // staging writes -> visible to the TMA store
@@ -269,7 +395,82 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 mbar_arrive(&tempty[buf]);
                 mbar_arrive(&sfull[sb]);
             }
+            if (++sb == NB) { sb = 0; sphase ^= 1u; }
             if (ew == 0 && lane == 0) trace_ev(p, 6, it);
+        }
+    } else if (F32 && warp >= kCvt0 && warp < kCvt0 + kNumCvtWarps) {
+        // ===================== fp32 -> space-to-depth codes (fused quantization) ===========
+        // The byte-coded halo X2 lives in a ring of NR = HR + Rt rows, every row stored twice
+        // (ring rows s and s + NR), so the HR rows of any tile are one contiguous window for
+        // the MMA descriptors.  A fresh tile (first of the CTA's run or of an image) quantizes
+        // its HR rows into ring rows 0..HR-1; a continuation tile only its Rt new rows (the run
+        // is contiguous: the others are the previous tile's), Rt ring rows further on.  Those
+        // rows last held rows of the tile two back (one back for a fresh tile), whose MMAs are
+        // waited for first.  Per tile: shifts, adds, selects -- no divisions.
+        const int ct = (warp - kCvt0) * 32 + lane;
+        const int NR = p.HR + p.Rt;
+        const uint32_t ring = smem_u32(smem + p.off_hx);
+        const uint32_t rowpx = static_cast<uint32_t>(p.Wh) * 16u;
+        const uint32_t mirror = static_cast<uint32_t>(NR) * rowpx;
+        const uint32_t zero = ring + 2u * mirror;        // 64 zero bytes after the ring
+        if (ct < 16) sts32(zero + 4u * ct, 0u);
+        const int tile_px = p.Rt * p.Wh;
+        // this thread's pixel of a continuation tile: new row nr, column jc
+        const bool has_new = ct < tile_px;
+        const int nr = has_new ? ct / p.Wh : 0, jc = has_new ? ct - nr * p.Wh : 0;
+        const uint32_t src_nr = 2u * static_cast<uint32_t>(nr) * static_cast<uint32_t>(p.f_rowbytes);
+        uint32_t coff[4];
+        const uint32_t cok = f32_s2d_offsets(p, jc, coff);
+        named_bar_sync(2, kNumCvtWarps * 32);           // the zero area is written
+        int base = 0;                                    // ring row of the tile's halo row 0
+        int g = 0;
+        RingPos rp, rp1, rp2;                            // tiles g, g-1, g-2
+        for (int tile = t_first; tile < t_end; tile += t_step, ++g, rp2 = rp1, rp1 = rp, rp.next(NS)) {
+            const int stage = rp.stage;
+            const int mt = p.fd_ntn.div(tile);
+            const int p0 = (mt - p.fd_tpi.div(mt) * p.tiles_per_img) * p.Rt;
+            const bool cont = tile != t_first && p0 != 0 && p.Rt < p.HR;
+            // MMAs still reading the ring rows rewritten here: tile g-2 (g-1 for a fresh tile)
+            if (cont ? g >= 2 : g >= 1) {
+                const RingPos &rb = cont ? rp2 : rp1;
+                mbar_wait(&hempty[rb.stage], rb.phase);
+            }
+            mbar_wait(&hfull[stage], rp.phase);
+            if (ct == 0) trace_ev(p, 8, g);
+            const uint32_t src = smem_u32(smem + p.off_hp + stage * p.hp_stage_bytes);
+            if (cont) {
+                base += p.Rt;
+                if (base >= NR) base -= NR;
+                if (has_new) {          // halo row HR - Rt + nr from staged rows 2 nr, 2 nr + 1
+                    int slot = base + p.HR - p.Rt + nr;
+                    if (slot >= NR) slot -= NR;
+                    uint32_t addr[4], w[4];
+                    f32_s2d_addr(src + src_nr, coff, cok, zero, addr);
+                    if (p.f_c == 3) f32_s2d_pixel<3>(p, addr, w);
+                    else f32_s2d_pixel<4>(p, addr, w);
+                    const uint32_t dst = ring + static_cast<uint32_t>(slot) * rowpx + 16u * static_cast<uint32_t>(jc);
+                    sts128(dst, w[0], w[1], w[2], w[3]);
+                    sts128(dst + mirror, w[0], w[1], w[2], w[3]);
+                }
+            } else {
+                base = 0;
+                for (int px = ct; px < p.HR * p.Wh; px += kNumCvtWarps * 32) {
+                    const int hr = px / p.Wh, j = px - (px / p.Wh) * p.Wh;
+                    uint32_t off[4], addr[4], w[4];
+                    const uint32_t ok = f32_s2d_offsets(p, j, off);
+                    f32_s2d_addr(src + 2u * static_cast<uint32_t>(hr) * static_cast<uint32_t>(p.f_rowbytes), off, ok,
+                                 zero, addr);
+                    if (p.f_c == 3) f32_s2d_pixel<3>(p, addr, w);
+                    else f32_s2d_pixel<4>(p, addr, w);
+                    const uint32_t dst = ring + static_cast<uint32_t>(hr) * rowpx + 16u * static_cast<uint32_t>(j);
+                    sts128(dst, w[0], w[1], w[2], w[3]);
+                    sts128(dst + mirror, w[0], w[1], w[2], w[3]);
+                }
+            }
+            fence_proxy_async_smem();                   // code rows -> visible to the MMA
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&hready[stage]);
+            if (ct == 0) trace_ev(p, 9, g);
         }
     } else if (IS4 && warp >= kCvt0 && warp < kCvt0 + kNumCvtWarps) {
         // ===================== int4 -> int8 plane widening =====================
@@ -279,10 +480,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         const uint32_t xo = p.x_sgn4 ? 0x88888888u : 0u;
         const int npix = p.HR * p.Wh;
         int g = 0;
-        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++g) {
-            const int stage = g % NS;
-            const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
-            mbar_wait(&hfull[stage], phase);
+        RingPos rp;
+        for (int tile = t_first; tile < t_end; tile += t_step, ++g, rp.next(NS)) {
+            const int stage = rp.stage;
+            mbar_wait(&hfull[stage], rp.phase);
             if (ct == 0) trace_ev(p, 8, g);
             const uint32_t src = smem_u32(smem + p.off_hp + stage * p.hp_stage_bytes);
             const uint32_t dst = smem_u32(smem + p.off_hx + stage * p.hx_stage_bytes);

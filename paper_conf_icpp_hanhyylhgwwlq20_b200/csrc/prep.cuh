@@ -13,36 +13,9 @@
 #include <cstdint>
 #include <cuda_bf16.h>
 #include "ptx.cuh"
+#include "quant.cuh"
 
 namespace qc {
-
-struct QuantParams {
-    const void *x;
-    void *y;
-    int64_t npix;
-    int32_t c, c_pad;
-    float inv_s;        // fl32(1/scale), computed on the host in fp32
-    float flo, fhi;     // qmin - z - 1, qmax - z + 1 (pre-clamp keeps the int conversion exact)
-    int32_t z, qmin, qmax;
-    int32_t bf16, bits;
-    int32_t fast;       // c == c_pad, c % 16 == 0, 16-byte aligned rows
-};
-
-__device__ __forceinline__ int32_t quantize_one(float x, const QuantParams &p) {
-    float t = __fmul_rn(x, p.inv_s);                 // one IEEE fp32 multiply, RNE
-    if (isnan(t)) return p.z;
-    t = fminf(fmaxf(t, p.flo), p.fhi);
-    const int32_t q = __float2int_rn(t) + p.z;       // round half to even
-    return min(p.qmax, max(p.qmin, q));
-}
-
-__device__ __forceinline__ float load_x(const QuantParams &p, int64_t i) {
-    if (p.bf16) {
-        const uint16_t b = static_cast<const uint16_t *>(p.x)[i];
-        return __uint_as_float(static_cast<uint32_t>(b) << 16);
-    }
-    return static_cast<const float *>(p.x)[i];
-}
 
 // One thread = 16 consecutive output elements (16 B of int8 or 8 B of int4).
 __global__ void __launch_bounds__(256) quantize_pack_kernel(const __grid_constant__ QuantParams p) {

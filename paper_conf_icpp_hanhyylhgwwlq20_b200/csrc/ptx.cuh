@@ -207,6 +207,9 @@ template <int N>
 __device__ __forceinline__ void bulk_wait() {
     asm volatile("cp.async.bulk.wait_group %0;" ::"n"(N) : "memory");
 }
+__device__ __forceinline__ void sts32(uint32_t addr, uint32_t a) {
+    asm volatile("st.shared.b32 [%0], %1;" ::"r"(addr), "r"(a) : "memory");
+}
 __device__ __forceinline__ void sts128(uint32_t addr, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
     asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d)
                  : "memory");
@@ -285,6 +288,24 @@ __device__ __forceinline__ void mma_i8_warp_lo(uint32_t d_tmem, uint32_t alo, ui
         "elect.sync _|e, 0xffffffff;\n\t"
         "@e tcgen05.mma.cta_group::1.kind::i8 [%0], da, db, %5, p;\n\t}" ::"r"(d_tmem),
         "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "r"(0), "r"(accumulate)
+        : "memory");
+}
+// Same, issued only when `active` is non-zero: a fully unrolled run of these has no branches,
+// so ptxas can move every MMA's register-to-uniform operand moves ahead of the issue chain
+// (branch-guarded MMAs each wait for their own moves: ~4x slower issue, measured).
+__device__ __forceinline__ void mma_i8_warp_lo_if(uint32_t d_tmem, uint32_t alo, uint32_t ahi, uint32_t blo,
+                                                  uint32_t bhi, uint32_t idesc, uint32_t accumulate,
+                                                  uint32_t active) {
+    asm volatile(
+        "{\n\t.reg .pred p, e, q;\n\t.reg .b64 da, db;\n\t"
+        "setp.ne.b32 p, %6, 0;\n\t"
+        "setp.ne.b32 q, %7, 0;\n\t"
+        "mov.b64 da, {%1, %2};\n\t"
+        "mov.b64 db, {%3, %4};\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "and.pred e, e, q;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::i8 [%0], da, db, %5, p;\n\t}" ::"r"(d_tmem),
+        "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "r"(accumulate), "r"(active)
         : "memory");
 }
 __device__ __forceinline__ void mma_commit_warp(uint64_t *bar) {

@@ -641,7 +641,9 @@ bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, bool ch
 }
 
 // ------------------------------------------------------------------ halo mode (stride 1)
-bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
+// f32_row_bytes > 0: the fused fp32-quantization stem (halo.cuh F32): the staging ring holds
+// the tile's 2*HR fp32 input rows of f32_row_bytes each instead of packed codes.
+bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f32_row_bytes = 0) {
     if (d->stride_h != 1 || d->stride_w != 1 || d->dil_h != 1 || d->dil_w != 1) return false;
     if (d->x_zero != 0 || !is_packed_out(d->y_t)) return false;
     const bool is4 = g.bits == 4;
@@ -681,21 +683,26 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     const int64_t num_tiles = static_cast<int64_t>(d->n) * tiles_per_img * n_tiles_n;
     if (num_tiles > INT32_MAX) return false;
     const uint32_t plane = static_cast<uint32_t>(HR * Wh * 16);
-    const uint32_t hx = static_cast<uint32_t>(align_up(static_cast<size_t>(nplanes) * plane, 1024));
-    const uint32_t hp = is4 ? static_cast<uint32_t>(align_up(static_cast<size_t>(nch) * plane, 1024)) : 0u;
+    // the fused fp32 stem keeps one ring of HR + Rt code rows, each stored twice, plus a
+    // 64-byte zero area (halo.cuh F32) instead of a code halo per stage
+    const uint32_t ringb = f32_row_bytes ? static_cast<uint32_t>(align_up(static_cast<size_t>(2 * (HR + Rt)) * Wh * 16 + 64, 1024)) : 0u;
+    const uint32_t hx = f32_row_bytes ? 0u : static_cast<uint32_t>(align_up(static_cast<size_t>(nplanes) * plane, 1024));
+    const uint32_t hp = f32_row_bytes ? static_cast<uint32_t>(align_up(static_cast<size_t>(2 * HR) * f32_row_bytes, 1024))
+                        : (is4 ? static_cast<uint32_t>(align_up(static_cast<size_t>(nch) * plane, 1024)) : 0u);
     const uint32_t bres = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * KG8, 1024));
     // output staging ring: 4 buffers when the halo ring keeps >= 3 stages, else 3, else 2
     int n_ystg = QC_MAX_YSTG;
     uint32_t ystg = 0, fixed = 0;
     for (;; --n_ystg) {
         ystg = static_cast<uint32_t>(n_ystg) * 128u * static_cast<uint32_t>(tile_row_bytes);
-        fixed = bres + ystg + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 2048u +
+        fixed = bres + ringb + ystg + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 2048u +
                 8u * static_cast<uint32_t>(d->r * d->s * nplanes);
         if (n_ystg == 2 || fixed + 3 * (hx + hp) <= 227u * 1024u) break;
     }
     if (fixed + 2 * (hx + hp) > 227u * 1024u) return false;
     int stages = static_cast<int>((227u * 1024u - fixed) / (hx + hp));
     stages = std::min(stages, 24);   // deep ring: the halo loads are latency-bound (~6 us each under load)
+    if (f32_row_bytes && (!tap_pair || stages < 3)) return false;   // (the ring reuse needs 3 stages)
     qc::ConvParams &p = pl->cp;
     std::memset(&p, 0, sizeof(p));
     p.M = static_cast<int32_t>(g.M);
@@ -710,9 +717,9 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     p.b_res_bytes = static_cast<uint32_t>(BN) * static_cast<uint32_t>(KG8);
     p.off_hx = bres;
     p.hx_stage_bytes = hx;
-    p.off_hp = bres + hx * stages;
+    p.off_hp = bres + (f32_row_bytes ? ringb : hx * stages);
     p.hp_stage_bytes = hp;
-    p.halo_tx = static_cast<uint32_t>(nch) * plane;
+    p.halo_tx = f32_row_bytes ? static_cast<uint32_t>(2 * HR) * f32_row_bytes : static_cast<uint32_t>(nch) * plane;
     // whole-row loads when one box row (Wh pixels) fits the 256-element limit as int64s and the
     // staged layout works without planes: the C = 16 stem (one plane) or 4-bit inputs (the
     // converter re-lays the packed pixels into planes)
@@ -744,7 +751,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl) {
     grid = std::max(grid / n_tiles_n * n_tiles_n, n_tiles_n);
     pl->kernel = QC_KERNEL_HALO;
     pl->grid = grid;
-    pl->threads = is4 ? 512 : 384;
+    pl->threads = (is4 || f32_row_bytes) ? 512 : 384;
     pl->BN = BN;
     pl->BM = qc::kBM;
     pl->n_tiles_n = n_tiles_n;
@@ -1205,6 +1212,132 @@ qc_status forward_impl(const qconv_desc *d, bool dequant, const void *x, const v
     return launch_plan(ex, pl, x_e, w_e, bias, mult, shift, dq, y, workspace, st);
 }
 
+// ------------------------------------------------------------------ fused quantization + conv
+// qconv2d_forward_quantize: float activations in.  The space-to-depth stem (stride 2, 4c <= 16)
+// runs the halo kernel with the quantization fused into its producer / converter warps
+// (halo.cuh F32); any other layer quantizes into the workspace, then runs qconv2d_forward.
+struct QExec {
+    bool fused;
+    Exec ex;                  // fused: the s2d exec descriptor; else the codes' exec descriptor
+    Plan pl;                  // fused: the halo plan with fp32 staging
+    qconv_desc dq;            // fallback: the descriptor of the quantized codes
+    size_t codes_bytes;       // fallback: quantized activations at the head of the workspace
+    size_t ws_total;
+};
+
+qc_status derive_qexec(const qconv_desc *d, qc_ftype xt, QExec *qx) {
+    if (!d) return QC_ERR_INVALID_ARG;
+    if (xt != QC_F32 && xt != QC_BF16) return QC_ERR_INVALID_ARG;
+    qconv_desc dv = *d;                      // codes of any 4-bit c live in bytes in the s2d form
+    dv.x_t = byte_container(d->x_t);
+    Geometry gv;
+    qc_status s = validate_desc(&dv, &gv, true);
+    if (s != QC_OK) return s;
+    if (!is_int_input(d->x_t)) return QC_ERR_INVALID_ARG;
+    const bool s2d_ok = d->stride_h == 2 && d->stride_w == 2 && d->dil_h == 1 && d->dil_w == 1 &&
+                        4 * d->c <= 16 && d->w_zero == nullptr && d->x_zero == 0 && xt == QC_F32 &&
+                        (static_cast<int64_t>(d->w) * d->c) % 4 == 0 && static_cast<int64_t>(d->w) * d->c <= 1024 &&
+                        is_packed_out(d->y_t);
+    qx->fused = false;
+    if (s2d_ok && check_overflow(d) == QC_OK) {
+        Exec &ex = qx->ex;
+        ex.d = d;
+        ex.gu = gv;
+        ex.e = s2d_of(d, gv);
+        if (validate_desc(&ex.e, &ex.g, false) == QC_OK && check_structure(&ex.e, ex.g) == QC_OK) {
+            ex.xform = XF_S2D;
+            ex.wprep = WP_S2D;
+            ex.wprep_needed = !d->w_prepared;
+            ex.prep_bytes = static_cast<size_t>(ex.g.w8_bytes);
+            ex.zx = ex.zw = false;
+            ex.off_w = ex.off_x = ex.off_zx = ex.off_cs = ex.off_x1 = 0;
+            ex.prologue = ex.wprep_needed ? 1 : 0;
+            ex.ws_total = ex.wprep_needed ? align_up(ex.prep_bytes, 256) : 0;
+            if (make_halo_plan(&ex.e, ex.g, &qx->pl, static_cast<uint32_t>(d->w) * d->c * 4u)) {
+                qx->fused = true;
+                qx->ws_total = ex.ws_total;
+                return QC_OK;
+            }
+        }
+    }
+    // fallback: codes in the workspace, then the ordinary forward
+    if (dtype_bits(d->x_t) == 4 && (d->c % 2)) return QC_ERR_UNSUPPORTED;   // no whole-byte code rows
+    qx->dq = *d;
+    s = derive_exec(&qx->dq, false, &qx->ex);
+    if (s != QC_OK) return s;
+    qx->codes_bytes = align_up(static_cast<size_t>(qx->ex.gu.x_bytes), 256);
+    qx->ws_total = qx->codes_bytes + qx->ex.ws_total;
+    return QC_OK;
+}
+
+qc_status launch_fused_stem(QExec &qx, const void *x, float in_scale, const void *w8, const int32_t *bias,
+                            const int32_t *mult, const int32_t *shift, void *y, cudaStream_t st) {
+    const Exec &ex = qx.ex;
+    const qconv_desc *d = ex.d;
+    const qconv_desc *e = &ex.e;
+    Plan &pl = qx.pl;
+    qc::ConvParams &p = pl.cp;
+    p.acc_lg = 0;
+    p.x_sgn4 = 0;
+    p.wsum = nullptr;
+    p.bias = bias;
+    p.mult = mult;
+    p.shift = shift;
+    p.y = y;
+    p.round_tfl = e->rounding == QC_ROUND_TFLITE ? 1 : 0;
+    p.q_inv_s = 1.0f / in_scale;
+    p.q_z = d->x_zero;
+    p.q_qmin = static_cast<int32_t>(dtype_min(d->x_t));
+    p.q_qmax = static_cast<int32_t>(dtype_max(d->x_t));
+    p.q_flo = static_cast<float>(p.q_qmin - p.q_z);     // exact integer bounds (halo.cuh f32_q)
+    p.q_fhi = static_cast<float>(p.q_qmax - p.q_z);
+    p.f_w = d->w;
+    p.f_c = d->c;
+    p.f_pad_h = d->pad_h;
+    p.f_pad_w = d->pad_w;
+    p.f_rowbytes = d->w * d->c * 4;
+    p.fd_pq = qc::make_fastdiv(static_cast<uint32_t>(p.PQ));
+    p.fd_q = qc::make_fastdiv(static_cast<uint32_t>(p.Q));
+    p.fd_ntn = qc::make_fastdiv(static_cast<uint32_t>(p.n_tiles_n));
+    p.fd_tpr = qc::make_fastdiv(1u);
+    p.fd_chunks = qc::make_fastdiv(1u);
+    p.fd_s = qc::make_fastdiv(static_cast<uint32_t>(std::max(1, p.S)));
+    p.fd_tpi = qc::make_fastdiv(static_cast<uint32_t>(std::max(1, p.tiles_per_img)));
+    alignas(64) CUtensorMap hm, bm, ym;
+    qc_status s = encode_halo_maps(e, ex.g, p, x, w8, y, &hm, &bm, &ym);
+    if (s != QC_OK) return s;
+    {   // fp32 input rows as raw 8-byte elements: [n][h][k pieces][row/k]; each row piece is one
+        // long contiguous TMA row (a 16-byte inner box would cost one request per 16 bytes);
+        // rows outside the image are zero-filled (= +0.0f, which quantizes to the zero point)
+        const Driver &drv = driver();
+        const cuuint64_t rowb = static_cast<cuuint64_t>(d->w) * d->c * 4;
+        cuuint64_t k = (rowb + 2047) / 2048;
+        while (rowb % (8 * k)) ++k;
+        const cuuint64_t piece = rowb / (8 * k);
+        cuuint64_t dims[4] = {piece, k, static_cast<cuuint64_t>(d->h), static_cast<cuuint64_t>(d->n)};
+        cuuint64_t strides[3] = {piece * 8, rowb, rowb * d->h};
+        cuuint32_t box[4] = {static_cast<cuuint32_t>(piece), static_cast<cuuint32_t>(k), 2, 1};   // one row pair
+        cuuint32_t es[4] = {1, 1, 1, 1};
+        if (piece > 256) return QC_ERR_UNSUPPORTED;
+        CUresult r = drv.tiled(&hm, CU_TENSOR_MAP_DATA_TYPE_INT64, 4, const_cast<void *>(x), dims, strides, box, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+    }
+    qc::Launch L;
+    L.grid = dim3(static_cast<unsigned>(pl.grid));
+    L.threads = pl.threads;
+    L.smem = pl.smem_bytes;
+    L.stream = st;
+    static const bool no_pdl = std::getenv("QC_NO_PDL") != nullptr;
+    L.pdl = !no_pdl;
+    debug_attach(p, st);
+    cudaError_t err = qc::launch_halo(L, false, out_kind(e->y_t), hm, bm, ym, p);
+    if (err != cudaSuccess) return cuda_fail(err);
+    debug_dump(p, st);
+    return QC_OK;
+}
+
 }  // namespace
 
 // ====================================================================== C ABI
@@ -1295,15 +1428,32 @@ qc_status qconv_quantize_pack(const void *x, qc_ftype xt, int64_t npix, int32_t 
     return QC_OK;
 }
 
+// Weight preparation of a descriptor whose activations only exist as floats for the fused
+// stem: 4-bit codes with an odd c have no packed NHWC form, but the space-to-depth operand holds
+// them in bytes, so the weights are prepared as for the byte-container view (same W2).
+static qc_status derive_exec_for_weights(const qconv_desc *d, Exec *ex, qconv_desc *tmp) {
+    qc_status s = derive_exec(d, true, ex);
+    if (s == QC_ERR_INVALID_ARG && d && is_int_input(d->x_t) && dtype_bits(d->x_t) == 4 && (d->c % 2)) {
+        *tmp = *d;
+        tmp->x_t = byte_container(d->x_t);
+        tmp->x_zero = 0;
+        s = derive_exec(tmp, true, ex);
+        if (s == QC_OK && ex->xform != XF_S2D) return QC_ERR_INVALID_ARG;
+    }
+    return s;
+}
+
 size_t qconv_prepared_weight_bytes(const qconv_desc *d) {
     Exec ex;
-    if (derive_exec(d, true, &ex) != QC_OK) return 0;
+    qconv_desc tmp;
+    if (derive_exec_for_weights(d, &ex, &tmp) != QC_OK) return 0;
     return ex.prep_bytes;
 }
 
 qc_status qconv_prepare_weights(const qconv_desc *d, const void *w, void *w_prep, void *stream) {
     Exec ex;
-    qc_status s = derive_exec(d, true, &ex);
+    qconv_desc tmp;
+    qc_status s = derive_exec_for_weights(d, &ex, &tmp);
     if (s != QC_OK) return s;
     if (!w || !w_prep) return QC_ERR_INVALID_ARG;
     if (!aligned16(w) || !aligned16(w_prep)) return QC_ERR_MISALIGNED;
@@ -1325,6 +1475,61 @@ qc_status qconv2d_forward(const qconv_desc *d, const void *x, const void *w, con
 qc_status qconv2d_forward_dequant(const qconv_desc *d, const void *x, const void *w, const int32_t *bias,
                                   const float *scale, void *y, void *workspace, size_t ws_bytes, void *stream) {
     return forward_impl(d, true, x, w, bias, nullptr, nullptr, scale, y, workspace, ws_bytes, stream);
+}
+
+size_t qconv2d_quantize_workspace_size(const qconv_desc *d, qc_ftype xt) {
+    QExec qx;
+    if (derive_qexec(d, xt, &qx) != QC_OK) return 0;
+    return qx.ws_total;
+}
+
+qc_status qconv2d_forward_quantize(const qconv_desc *d, const void *x, qc_ftype xt, float in_scale,
+                                   const void *w, const int32_t *bias, const int32_t *multiplier,
+                                   const int32_t *shift, void *y, void *workspace, size_t ws_bytes,
+                                   void *stream) {
+    QExec qx;
+    qc_status s = derive_qexec(d, xt, &qx);
+    if (s != QC_OK) return s;
+    if (!x || !w || !y) return QC_ERR_INVALID_ARG;
+    if (!(in_scale > 0.0f) || !std::isfinite(in_scale)) return QC_ERR_INVALID_ARG;
+    if (qx.ws_total > 0 && (!workspace || ws_bytes < qx.ws_total)) return QC_ERR_WORKSPACE;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (!qx.fused)
+        if (!aligned16(x) || (workspace && !aligned16(workspace))) return QC_ERR_MISALIGNED;
+    if (qx.fused) {
+        if (is_packed_out(d->y_t) && (!multiplier || !shift)) return QC_ERR_INVALID_ARG;
+        if (!aligned16(x) || !aligned16(w) || !aligned16(y) || (bias && !aligned16(bias)) ||
+            (multiplier && !aligned16(multiplier)) || (shift && !aligned16(shift)))
+            return QC_ERR_MISALIGNED;
+        const void *w8 = w;
+        if (qx.ex.wprep_needed) {
+            s = prepare_weights_exec(qx.ex, w, workspace, st);
+            if (s != QC_OK) return s;
+            w8 = workspace;
+        }
+        return launch_fused_stem(qx, x, in_scale, w8, bias, multiplier, shift, y, st);
+    }
+    uint8_t *codes = static_cast<uint8_t *>(workspace);
+    s = qconv_quantize_pack(x, xt, static_cast<int64_t>(d->n) * d->h * d->w, d->c, d->c, in_scale, d->x_zero,
+                            d->x_t, codes, stream);
+    if (s != QC_OK) return s;
+    return forward_impl(&qx.dq, false, codes, w, bias, multiplier, shift, nullptr, y, codes + qx.codes_bytes,
+                        ws_bytes - qx.codes_bytes, stream);
+}
+
+qc_status qconv_debug_plan_quantize(const qconv_desc *d, qc_ftype xt, qconv_plan *out) {
+    if (!out) return QC_ERR_INVALID_ARG;
+    QExec qx;
+    qc_status s = derive_qexec(d, xt, &qx);
+    if (s != QC_OK) return s;
+    if (qx.fused) {
+        fill_plan_out(qx.ex, qx.pl, out);
+        out->prologue = qx.ex.prologue;
+        return QC_OK;
+    }
+    s = qconv_debug_plan(&qx.dq, out);
+    if (s == QC_OK) out->prologue |= 16;      // + the separate quantize launch
+    return s;
 }
 
 qc_status qconv_debug_plan(const qconv_desc *d, qconv_plan *out) {

@@ -22,12 +22,15 @@ os.environ["QC_TRACE"] = out
 L = tr.layers[j]
 print(L["name"], L["plan"])
 for _ in range(2):
-    tr.qc.qconv2d_forward(L["desc"], L["x"], L["w"], L["bias"], L["m"], L["n"], y=L["y"])
+    if j == 0:
+        tr.qc.qconv2d_forward_quantize(L["desc"], tr.x_float, tr.s_in, L["w"], L["bias"], L["m"], L["n"], y=L["y"])
+    else:
+        tr.qc.qconv2d_forward(L["desc"], L["x"], L["w"], L["bias"], L["m"], L["n"], y=L["y"])
 torch.cuda.synchronize()
 t = np.fromfile(out, dtype=np.uint64).reshape(-1, 16, 1024).astype(np.int64)[-1]
 t0 = min(v for v in t.reshape(-1) if v > 0)
 names = {0: "prod", 2: "mma_acc_free", 3: "mma_in", 1: "mma_fenced", 11: "mma_issued", 12: "commit_empty",
-         4: "commit_tfull", 5: "epi_acc_full", 6: "epi_done", 7: "store", 8: "cvt_in", 9: "cvt_done"}
+         4: "commit_tfull", 5: "epi_acc_full", 6: "epi_done", 7: "store", 8: "cvt_in", 10: "epi_stg_free", 13: "epi_ld_done", 14: "epi_requant_done", 9: "cvt_done"}
 for ev, nm in names.items():
     row = t[ev][t[ev] > 0] - t0
     if len(row) > 1:

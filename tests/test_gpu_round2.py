@@ -331,3 +331,63 @@ def test_autotune_records_an_exact_plan():
     torch.cuda.synchronize()
     _assert_same(y.cpu().numpy(), ref, "autotuned")
     qc.qconv_plan_set(d, None)
+
+
+@pytest.mark.parametrize("bits", [8, 4])
+@pytest.mark.parametrize("n_img,relu", [(2, True), (1, False)])
+def test_forward_quantize_fused_stem(bits, n_img, relu):
+    """qconv2d_forward_quantize on the C = 3 stem: one kernel quantizes the fp32 rows (Z4) into
+    its space-to-depth operand tile; compared with oracle quantize (+ a zero-point channel) then
+    the oracle's direct 7x7/s2 conv.  Inputs include NaN, +-inf and exact quantization ties."""
+    cs = ConvShape("stem", n_img, 224, 224, 3, 64, 7, 7, 2, 3)
+    rng = np.random.default_rng(60 + bits + n_img)
+    xf = float_image(rng, (n_img, 224, 224, 3))
+    s_x = 3.0 / 15 if bits == 4 else 3.0 / 255
+    xf.reshape(-1)[:6] = [np.nan, np.inf, -np.inf, 0.5 * s_x, 1.5 * s_x, 2.5 * s_x]
+    xt = U4 if bits == 4 else U8
+    li = make_layer_inputs(cs, bits, seed=3 + bits, c_store=4, relu=relu, signed_out=not relu)
+    li.x_bytes = oracle.quantize(xf, s_x, 0, xt, c_pad=4)
+    m, n = oracle.requant_params(li.s_x, li.s_w, li.s_y)
+    ref = oracle.conv2d_layer(li, mult=m, shift=n)
+    d = qc.make_desc(n_img, 224, 224, 3, 64, 7, 7, stride=2, pad=3, x_t=xt, w_t=S8, y_t=li.y_t,
+                     clamp_lo=li.clamp_lo, clamp_hi=li.clamp_hi)
+    w = torch.from_numpy(np.ascontiguousarray(pack_codes(li.w_codes[..., :3], S8))).to(DEV)
+    b, mm, nn = (torch.from_numpy(a).to(DEV) for a in (li.bias, m, n))
+    y = qc.qconv2d_forward_quantize(d, torch.from_numpy(xf).to(DEV), s_x, w, b, mm, nn)
+    torch.cuda.synchronize()
+    _assert_same(y.cpu().numpy(), ref, "fused stem (unprepared weights)")
+    wp = qc.qconv_prepare_weights(d, w)
+    d.w_prepared = 1
+    assert qc._lib().qconv2d_quantize_workspace_size(d, qc.QC_F32) == 0     # one kernel, no workspace
+    y = qc.qconv2d_forward_quantize(d, torch.from_numpy(xf).to(DEV), s_x, wp, b, mm, nn)
+    torch.cuda.synchronize()
+    _assert_same(y.cpu().numpy(), ref, "fused stem (prepared weights)")
+
+
+@pytest.mark.parametrize("cs,bits,x_zero,bf16", [
+    (ConvShape("q1", 2, 9, 11, 64, 48, 3, 3, 1, 1), 8, 0, False),
+    (ConvShape("q2", 2, 12, 12, 32, 64, 1, 1), 4, 3, True),
+    (ConvShape("q3", 1, 32, 32, 3, 16, 7, 7, 2, 3), 8, 5, False),      # stem shape, x_zero: two launches
+], ids=lambda v: getattr(v, "name", str(v)))
+def test_forward_quantize_general(cs, bits, x_zero, bf16):
+    """Descriptors outside the fused stem case: quantize into the workspace, then the conv."""
+    rng = np.random.default_rng(cs.c + bits)
+    xf = rng.normal(0.5, 1.0, size=(cs.n, cs.h, cs.w, cs.c)).astype(np.float32)
+    xt = U4 if bits == 4 else U8
+    s_x = 0.11
+    xtensor = torch.from_numpy(xf)
+    if bf16:
+        xtensor = xtensor.to(torch.bfloat16)
+        host = xtensor.view(torch.int16).numpy().view(np.uint16)
+    else:
+        host = xf
+    li = make_layer_inputs(cs, bits, seed=cs.k, relu=True, x_zero=x_zero)
+    li.x_bytes = oracle.quantize(host, s_x, x_zero, xt, bf16=bf16)
+    m, n = oracle.requant_params(li.s_x, li.s_w, li.s_y)
+    ref = oracle.conv2d_layer(li, mult=m, shift=n)
+    d = _desc(li)
+    b, mm, nn = (torch.from_numpy(a).to(DEV) for a in (li.bias, m, n))
+    y = qc.qconv2d_forward_quantize(d, xtensor.to(DEV).contiguous(), s_x,
+                                    torch.from_numpy(li.w_bytes).to(DEV), b, mm, nn)
+    torch.cuda.synchronize()
+    _assert_same(y.cpu().numpy(), ref, cs.name)
