@@ -288,6 +288,15 @@ __device__ __forceinline__ void epi_requant16(const ConvParams &p, uint32_t (&v)
     }
 }
 
+// Position in an NS-stage mbarrier ring (stage, phase parity), advanced without divisions.
+struct RingPos {
+    int stage = 0;
+    uint32_t phase = 0;
+    __device__ __forceinline__ void next(int ns) {
+        if (++stage == ns) { stage = 0; phase ^= 1u; }
+    }
+};
+
 // Pack and store outputs v[H .. H+16) of one row = output channels [kc, kc+16) straight
 // to global memory (int32 and float outputs, and packed outputs without a TMA store map).
 template <int OUT, int H>

@@ -98,22 +98,14 @@ __device__ __forceinline__ void f32_s2d_addr(uint32_t rows, const uint32_t (&off
     for (int blk = 0; blk < 4; ++blk) addr[blk] = (ok >> blk) & 1u ? rows + off[blk] : zero;
 }
 
-// Position in an NS-stage mbarrier ring (stage, phase parity), advanced without divisions.
-struct RingPos {
-    int stage = 0;
-    uint32_t phase = 0;
-    __device__ __forceinline__ void next(int ns) {
-        if (++stage == ns) { stage = 0; phase ^= 1u; }
-    }
-};
-
 template <bool IS4, int OUT, bool F32 = false>
 __global__ void __launch_bounds__((IS4 || F32) ? 512 : 384, 1)
 qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap bmap,
                   const __grid_constant__ CUtensorMap ymap, const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                                ~uintptr_t(1023));
+    // 1024-byte aligned base by pointer arithmetic on the shared array itself (no integer round
+    // trip): the compiler keeps it in the shared window, so every smem_u32() below is one add
+    uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
     const int NS = p.stages;

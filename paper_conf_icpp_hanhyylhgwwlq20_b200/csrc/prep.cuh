@@ -415,8 +415,9 @@ __global__ void qconv_debug_im2col_kernel(const __grid_constant__ CUtensorMap xm
                                           int32_t w, int32_t h, int32_t n, uint16_t ow,
                                           uint16_t oh, uint32_t bytes, uint8_t *out) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                                ~uintptr_t(1023));
+    // 1024-byte aligned base by pointer arithmetic on the shared array itself (no integer round
+    // trip): the compiler keeps it in the shared window, so every smem_u32() below is one add
+    uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     __shared__ __align__(8) uint64_t bar;
     if (threadIdx.x == 0) {
         mbar_init(&bar, 1);

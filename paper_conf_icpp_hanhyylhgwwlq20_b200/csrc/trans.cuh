@@ -135,8 +135,9 @@ __global__ void __launch_bounds__(IS4 ? kTThreads4 : kTThreads8, 1)
 qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__ CUtensorMap wmap,
                const __grid_constant__ CUtensorMap ymap, const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                                ~uintptr_t(1023));
+    // 1024-byte aligned base by pointer arithmetic on the shared array itself (no integer round
+    // trip): the compiler keeps it in the shared window, so every smem_u32() below is one add
+    uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
     const int NS = p.stages;
@@ -236,6 +237,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         // whole warp runs the loop, one elected lane issues (see conv_fwd.cuh)
         {
             int it = 0, g = 0;
+            RingPos rp;
             const uint32_t sbo = 8u * static_cast<uint32_t>(p.BK);
             const int ksteps = p.BK / 32;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
@@ -246,10 +248,9 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 tc_fence_after();
                 if (lane == 0) trace_ev(p, 2, it);
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * BNp);
-                for (int kb = 0; kb < p.num_kb; ++kb, ++g) {
-                    const int stage = g % NS;
-                    const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
-                    mbar_wait(IS4 ? &aready[stage] : &full[stage], phase);
+                for (int kb = 0; kb < p.num_kb; ++kb, ++g, rp.next(NS)) {
+                    const int stage = rp.stage;
+                    mbar_wait(IS4 ? &aready[stage] : &full[stage], rp.phase);
                     __syncwarp();
                     tc_fence_after();
                     if (lane == 0) trace_ev(p, 3, g);
@@ -297,10 +298,16 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         TChan ce{}, co{};
         int mode = 2;
         int it = 0;
+        // channel tile of the CTA's current tile, advanced without divisions
+        const int ntn = p.n_tiles_n;
+        const int cstep = static_cast<int>(gridDim.x) % ntn;
+        int cm = static_cast<int>(blockIdx.x) % ntn;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
-            const int c0 = (tile % p.n_tiles_n) * BMc;
+            const int c0 = cm * BMc;
+            cm += cstep;
+            if (cm >= ntn) cm -= ntn;
             if (c0 != cached_c0) {
                 const int ke = c0 + 2 * pair, ko = ke + 1;
                 int nee, neo;
@@ -353,11 +360,11 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         const uint32_t sw = static_cast<uint32_t>(p.sw_mask);
         const uint32_t bkb = static_cast<uint32_t>(p.BK);
         int g = 0;
+        RingPos rp;
         for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
-            for (int kb = 0; kb < p.num_kb; ++kb, ++g) {
-                const int stage = g % NS;
-                const uint32_t phase = static_cast<uint32_t>(g / NS) & 1u;
-                mbar_wait(&full[stage], phase);
+            for (int kb = 0; kb < p.num_kb; ++kb, ++g, rp.next(NS)) {
+                const int stage = rp.stage;
+                mbar_wait(&full[stage], rp.phase);
                 if (ct == 0) trace_ev(p, 8, g);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
                 const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);

@@ -10,6 +10,9 @@ import bench  # noqa: E402
 bits = int(sys.argv[1]) if len(sys.argv) > 1 else 4
 j = int(sys.argv[2]) if len(sys.argv) > 2 else 0
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 3
+from paper_conf_icpp_hanhyylhgwwlq20_b200 import tuning  # noqa: E402
+tuning.load_plans(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "plans",
+                               f"resnet50_trunk_a{bits}_b256.json"))
 tr = bench.Trunk(bits, 256, torch.device("cuda", 0))
 L = tr.layers[j]
 print(L["name"], L["plan"])
