@@ -35,6 +35,9 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t by
                  "r"(bytes)
                  : "memory");
 }
+__device__ __forceinline__ void mbar_arrive_a(uint32_t addr) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(addr) : "memory");
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -70,10 +73,23 @@ __device__ __forceinline__ bool mbar_try_wait_sleep(uint32_t addr, uint32_t pari
 // issue slots from working warps.  A wait longer than ~4 s traps (a protocol
 // bug becomes a launch error instead of a hang).
 #ifndef QC_WAIT_SLEEP
-#define QC_WAIT_SLEEP 0
+#define QC_WAIT_SLEEP 1
 #endif
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
     const uint32_t a = smem_u32(bar);
+    if (mbar_try_wait(a, parity)) return;
+    uint64_t t0 = 0;
+    uint32_t it = 0;
+    while (!(QC_WAIT_SLEEP ? mbar_try_wait_sleep(a, parity) : mbar_try_wait(a, parity))) {
+        if ((++it & 63u) == 0) {
+            const uint64_t t = globaltimer_ns();
+            if (t0 == 0) t0 = t;
+            else if (t - t0 > 4000000000ull) __trap();
+        }
+    }
+}
+
+__device__ __forceinline__ void mbar_wait_a(uint32_t a, uint32_t parity) {
     if (mbar_try_wait(a, parity)) return;
     uint64_t t0 = 0;
     uint32_t it = 0;
