@@ -4,9 +4,11 @@
 Default workload = BASELINE configs[4] ("C5"): the ResNet-50 conv trunk at A4W4, global
 batch 256, batch-sharded over the GPUs (strong scaling: 256/G images per GPU; `--batch B`
 gives weak scaling with B images per GPU).  One step = the whole hot path (SURVEY.md 8(a)
-rows a1, a3-a6) over one batch: the fused fp32 quantize + space-to-depth of the stem input,
-then the 53 ResNet-50 conv layers (qconv2d_forward: implicit GEMM on tcgen05 tensor cores
-with bias / re-quantization / ReLU / packing fused), chained in network order.  Weight and
+rows a1, a3-a6) over one batch: the 53 ResNet-50 conv layers chained in network order --
+the stem takes the fp32 image (qconv2d_forward_quantize: the quantization to codes runs
+inside the stem kernel, space-to-depth form), the other 52 take the previous layer's packed
+codes (qconv2d_forward: implicit GEMM on tcgen05 tensor cores with bias / re-quantization /
+ReLU / packing fused).  Weight and
 parameter preparation (row a2) happens once, off the timed path; with N GPUs rank 0's
 weights are broadcast once over NCCL -- the only collective (row e).
 

@@ -6,7 +6,7 @@ cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 for b in 4 8; do
   timeout 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
-    -k regex:"qconv|quantize_s2d" -s 54 -c 54 --csv --log-file gpurun_out/${TAG}_launches_a$b.csv \
+    -k regex:"qconv" -s 53 -c 53 --csv --log-file gpurun_out/${TAG}_launches_a$b.csv \
     python bench.py --bits $b --profile-steps 1 --warmup 1 > gpurun_out/${TAG}_ncu_launch_a$b.log 2>&1
   python scripts/prof_launches.py gpurun_out/${TAG}_launches_a$b.csv ${TAG}_a$b $b 256
 done
