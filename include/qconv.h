@@ -235,6 +235,8 @@ qc_status qconv2d_forward_quantize(const qconv_desc *d, const void *x, qc_ftype 
  *            QC_KERNEL_PAIR     im2col on a 2-CTA cluster (tcgen05 cta_group::2, M = 256)
  *            QC_KERNEL_HALO     stride-1 halo tiles, weights resident in shared memory
  *            QC_KERNEL_CHANNEL  1x1 convs, channel-major (output channels on TMEM lanes)
+ *            QC_KERNEL_HALO_T   stride-1 halo tiles, channel-major (K = 64 output channels on
+ *                               TMEM lanes, up to 256 pixels per tile)
  *   bn     : output channels per tile (IM2COL/PAIR: 16..256; CHANNEL: 64 or 128; HALO: K)
  * qconv_debug_plan fills every field of the plan qconv2d_forward would launch for `d`
  * (after any qconv_plan_set choice); the pre-kernels (weight preparation, activation
@@ -250,7 +252,7 @@ qc_status qconv2d_forward_quantize(const qconv_desc *d, const void *x, qc_ftype 
  * mean time in `best_us`.  It writes `y` (every candidate gives the same bytes).
  */
 typedef enum { QC_KERNEL_AUTO = 0, QC_KERNEL_IM2COL = 1, QC_KERNEL_PAIR = 2, QC_KERNEL_HALO = 3,
-               QC_KERNEL_CHANNEL = 4 } qc_kernel;
+               QC_KERNEL_CHANNEL = 4, QC_KERNEL_HALO_T = 5 } qc_kernel;
 typedef struct {
     int32_t kernel;           /* qc_kernel */
     int32_t bn;               /* output channels per tile */

@@ -22,8 +22,8 @@ _SO = os.path.join(_PKG, "libqconv.so")
 QC_U4, QC_S4, QC_U8, QC_S8, QC_S32, QC_F32_OUT, QC_BF16_OUT = 0, 1, 2, 3, 4, 5, 6
 QC_F32, QC_BF16 = 0, 1
 QC_ROUND_SINGLE, QC_ROUND_TFLITE = 0, 1
-QC_KERNEL_AUTO, QC_KERNEL_IM2COL, QC_KERNEL_PAIR, QC_KERNEL_HALO, QC_KERNEL_CHANNEL = 0, 1, 2, 3, 4
-KERNEL_NAMES = {0: "auto", 1: "im2col", 2: "pair", 3: "halo", 4: "channel"}
+QC_KERNEL_AUTO, QC_KERNEL_IM2COL, QC_KERNEL_PAIR, QC_KERNEL_HALO, QC_KERNEL_CHANNEL, QC_KERNEL_HALO_T = 0, 1, 2, 3, 4, 5
+KERNEL_NAMES = {0: "auto", 1: "im2col", 2: "pair", 3: "halo", 4: "channel", 5: "halo_t"}
 _BITS = {QC_U4: 4, QC_S4: 4, QC_U8: 8, QC_S8: 8, QC_S32: 32, QC_F32_OUT: 32, QC_BF16_OUT: 16}
 _RANGE = {QC_U4: (0, 15), QC_S4: (-8, 7), QC_U8: (0, 255), QC_S8: (-128, 127),
           QC_S32: (-(2 ** 31), 2 ** 31 - 1)}
@@ -429,7 +429,7 @@ __all__ = ["qconv_quantize_pack", "qconv_requant_params", "qconv_prepare_weights
            "qconv2d_forward_dequant", "qconv2d_forward_quantize", "qconv_debug_plan", "qconv_debug_plan_quantize", "qconv_plan_candidates",
            "qconv_plan_set", "qconv_plan_clear", "qconv_autotune", "qconv_plan",
            "QC_F32_OUT", "QC_BF16_OUT", "QC_ROUND_SINGLE", "QC_ROUND_TFLITE",
-           "QC_KERNEL_AUTO", "QC_KERNEL_IM2COL", "QC_KERNEL_PAIR", "QC_KERNEL_HALO",
+           "QC_KERNEL_AUTO", "QC_KERNEL_IM2COL", "QC_KERNEL_PAIR", "QC_KERNEL_HALO", "QC_KERNEL_HALO_T",
            "QC_KERNEL_CHANNEL",
            "qconv_s2d_desc", "qconv_quantize_pack_s2d", "qconv_prepare_weights_s2d",
            "qconv_prepared_weight_bytes", "qconv2d_workspace_size", "qconv2d_forward",

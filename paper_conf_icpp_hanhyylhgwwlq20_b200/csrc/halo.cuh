@@ -19,6 +19,7 @@
 #pragma once
 #include "epilogue.cuh"
 #include "quant.cuh"
+#include "trans.cuh"
 
 namespace qc {
 
@@ -98,8 +99,14 @@ __device__ __forceinline__ void f32_s2d_addr(uint32_t rows, const uint32_t (&off
     for (int blk = 0; blk < 4; ++blk) addr[blk] = (ok >> blk) & 1u ? rows + off[blk] : zero;
 }
 
-template <bool IS4, int OUT, bool F32 = false>
-__global__ void __launch_bounds__((IS4 || F32) ? 512 : 384, 1)
+// CM = channel-major variant (K = 64): the UMMA computes D^T = W * X^T with M = 64 output
+// channels (the resident weights, rows permuted so TMEM lanes l and l+8 hold a channel pair)
+// and N = Rt * Wh pixels (the halo, rows padded to Wh = a multiple of 8, N <= 256); the
+// epilogue is the channel-pair epilogue of trans.cuh (constants in registers, ~3 instructions
+// per output) with 16 warps, and the storer writes one output row per TMA store.
+template <bool IS4, int OUT, bool F32 = false, bool CM = false>
+__global__ void __launch_bounds__(CM ? ((IS4 || F32) ? kTThreads4 : kTThreads8)
+                                     : ((IS4 || F32) ? 512 : 384), 1)
 qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constant__ CUtensorMap bmap,
                   const __grid_constant__ CUtensorMap ymap, const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -129,9 +136,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
     // ids (B300_MICROARCH "hi-wid-first"), and the MMA warp's issue loop (8-18 MMAs per tile)
     // is on the kernel's critical path, so it must not wait behind epilogue instructions.
     constexpr int kEpi0 = 0;
-    constexpr int kCvt0 = kNumEpiWarps;
+    constexpr int kNEpi = CM ? kTEpiWarps : kNumEpiWarps;
+    constexpr int kCvt0 = kNEpi;
     constexpr bool kCvt = IS4 || F32;                // converter warps present
-    constexpr int kCtl0 = kNumEpiWarps + (kCvt ? kNumCvtWarps : 0);
+    constexpr int kCtl0 = kNEpi + (kCvt ? kNumCvtWarps : 0);
     constexpr int kProd = kCtl0, kStorer = kCtl0 + 1, kMma = kCtl0 + 3;
     griddep_launch_dependents();
     if (warp == kProd && lane == 0) {
@@ -145,10 +153,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(&tfull[i], 1);
-            mbar_init(&tempty[i], kNumEpiWarps);
+            mbar_init(&tempty[i], kNEpi);
         }
         for (int i = 0; i < kMaxYstg; ++i) {
-            mbar_init(&sfull[i], kNumEpiWarps);
+            mbar_init(&sfull[i], kNEpi);
             mbar_init(&sfree[i], 1);
         }
         mbar_init(bfull, 1);
@@ -183,7 +191,11 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 const int img = p.fd_tpi.div(mt);
                 const int p0 = (mt - img * p.tiles_per_img) * p.Rt;
                 mbar_wait(&sfull[b], bphase);
-                {
+                if (CM) {   // one store per output row: staging row = accumulator column
+                    for (int rr = 0; rr < p.Rt; ++rr)
+                        tma_store_4d(&ymap, smem + p.off_ystg + b * p.ystg_bytes + rr * p.Wh * p.y_gw, 0, 0,
+                                     p0 + rr, img);
+                } else {
                     constexpr int kBits = (OUT == OUT_U4 || OUT == OUT_S4) ? 4 : 8;
                     for (int gi = 0; gi < p.n_ygroups; ++gi)
                         tma_store_4d(&ymap, smem + p.off_ystg + b * p.ystg_bytes + gi * 128 * p.y_gw,
@@ -207,7 +219,11 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             // stream (weight preparation, or the caller's own kernels): wait for it first
             griddep_wait();
             if (leader) mbar_arrive_expect_tx(bfull, p.b_res_bytes);
-            if (leader) tma_load_3d(smem + p.off_bres, &bmap, bfull, 0, n0, 0);
+            if (CM) {   // permuted 5-D view (channel pairs on TMEM lanes l, l+8); K = 64: n0 = 0
+                if (leader) tma_load_5d(smem + p.off_bres, &bmap, bfull, 0, 0, 0, 0, 0);
+            } else {
+                if (leader) tma_load_3d(smem + p.off_bres, &bmap, bfull, 0, n0, 0);
+            }
             int g = 0;
             RingPos rp;
             for (int tile = t_first; tile < t_end; tile += t_step, ++g, rp.next(NS)) {
@@ -283,7 +299,7 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 __syncwarp();
                 tc_fence_after();
                 if (leader) trace_ev(p, 1, it);
-                const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * p.BN);
+                const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * (CM ? 256 : p.BN));
                 uint32_t alo0 = static_cast<uint32_t>(adesc_st) +
                                 ((static_cast<uint32_t>(stage) * p.hx_stage_bytes) >> 4);
                 if (F32) {   // the tile's window of the converter's code-row ring (same sequence)
@@ -302,9 +318,14 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 // shared memory per 52 cycles (scripts/micro/mma_bench3.cu); guarded by a branch
                 // each, the issue chain paced them at ~150-270.
 #pragma unroll
-                for (int i = 0; i < kHaloMaxMMA; ++i)
-                    mma_i8_warp_lo_if(d_tmem, alo0 + aoff[i], ahi, blo0 + boff[i], bhi, p.idesc, i > 0 ? 1u : 0u,
-                                      i < nmma ? 1u : 0u);
+                for (int i = 0; i < kHaloMaxMMA; ++i) {
+                    if (CM)      // A = the weights (M = 64 channels), B = the halo (N pixels)
+                        mma_i8_warp_lo_if(d_tmem, blo0 + boff[i], bhi, alo0 + aoff[i], ahi, p.idesc,
+                                          i > 0 ? 1u : 0u, i < nmma ? 1u : 0u);
+                    else
+                        mma_i8_warp_lo_if(d_tmem, alo0 + aoff[i], ahi, blo0 + boff[i], bhi, p.idesc,
+                                          i > 0 ? 1u : 0u, i < nmma ? 1u : 0u);
+                }
                 if (leader) trace_ev(p, 11, it);
                 mma_commit_warp(&hempty[stage]);
                 if (leader) trace_ev(p, 12, it);
@@ -313,7 +334,70 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 if (++stage == NS) { stage = 0; phase ^= 1u; }
             }
         }
-    } else if (warp >= kEpi0 && warp < kEpi0 + kNumEpiWarps) {
+    } else if (CM && warp >= kEpi0 && warp < kEpi0 + kNEpi) {
+        // ===================== channel-major epilogue (trans.cuh, M = 64) =====================
+        // warp w: TMEM lanes 32 (w % 4) .. +15 (output channels 16 (w % 4) .. +15 as 8 pairs,
+        // lanes l and l+8 = channels 2i, 2i+1 of the permuted weight rows), accumulator columns
+        // 64 (w / 4) .. +63 (tile pixels; staging row = column, 8-row-aligned output rows)
+        griddep_wait();                                   // params written in-stream
+        const int ew = warp - kEpi0;
+        const int quarter = warp & 3;
+        const int sub = ew >> 2;
+        constexpr bool kInt4 = (OUT == OUT_U4 || OUT == OUT_S4);
+        constexpr int kRowBytes = 64 * (kInt4 ? 4 : 8) / 8;
+        constexpr int kGMask = kRowBytes >= 128 ? 7 : (kRowBytes == 64 ? 3 : 1);
+        const uint32_t lane_base = 32u * static_cast<uint32_t>(quarter);
+        const int col_begin = sub * 64;
+        const int pair = 8 * quarter + (lane >> 2);
+        const uint32_t boff = static_cast<uint32_t>(kInt4 ? pair : 2 * pair);
+        const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
+        TChan ce{}, co{};
+        int mode;
+        {
+            const int ke = 2 * pair, ko = ke + 1;
+            int nee, neo;
+            bool be, bo;
+            t_chan_params(p, ke, ke < p.K, ce, nee, be);
+            t_chan_params(p, ko, ko < p.K, co, neo, bo);
+            const unsigned act = 0xffffffffu;
+            const bool all_fast = __ballot_sync(act, be && bo && nee >= 33 && nee <= 52 && neo >= 33 && neo <= 52) == act;
+            const bool all_mid = __ballot_sync(act, be && bo && nee >= 20 && nee <= 50 && neo >= 20 && neo <= 50 &&
+                                                        mid_multiplier_ok(ce.m) && mid_multiplier_ok(co.m)) == act;
+            mode = all_fast ? 0 : (all_mid ? 1 : 2);
+            if (mode == 1) {
+                const int T = max(33, __reduce_max_sync(act, max(nee, neo)));
+                t_chan_mid(p, ce, nee, T);
+                t_chan_mid(p, co, neo, T);
+            }
+        }
+        const uint32_t taddr0 = tmem_base + (lane_base << 16) + static_cast<uint32_t>(col_begin);
+        const int row0 = col_begin + 2 * (lane & 3);
+        int it = 0;
+        int sb = 0;
+        uint32_t sphase = 0;
+        for (int tile = t_first; tile < t_end; tile += t_step, ++it) {
+            const int buf = it & 1;
+            const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
+            mbar_wait(&tfull[buf], acc_phase);
+            tc_fence_after();
+            if (ew == 0 && lane == 0) trace_ev(p, 5, it);
+            mbar_wait(&sfree[sb], sphase ^ 1u);
+            const uint32_t ystg = ystg_base + static_cast<uint32_t>(sb) * p.ystg_bytes;
+            uint32_t va[32];
+            tmem_ld_16x256b_x8(taddr0 + static_cast<uint32_t>(buf * 256), va);
+            tmem_wait_ld_regs(va);
+            t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, va, ystg, row0, boff);
+            tc_fence_before();
+            fence_proxy_async_smem();                 // staging writes -> visible to the TMA store
+            __syncwarp();
+            if (lane == 0) {
+                mbar_arrive(&tempty[buf]);
+                mbar_arrive(&sfull[sb]);
+            }
+            if (++sb == NB) { sb = 0; sphase ^= 1u; }
+            if (ew == 0 && lane == 0) trace_ev(p, 6, it);
+        }
+    } else if (!CM && warp >= kEpi0 && warp < kEpi0 + kNumEpiWarps) {
         // ===================== epilogue =====================
         griddep_wait();                                   // params written in-stream
         const int ew = warp - kEpi0;
@@ -407,12 +491,20 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         const uint32_t zero = ring + 2u * mirror;        // 64 zero bytes after the ring
         if (ct < 16) sts32(zero + 4u * ct, 0u);
         const int tile_px = p.Rt * p.Wh;
-        // this thread's pixel of a continuation tile: new row nr, column jc
-        const bool has_new = ct < tile_px;
-        const int nr = has_new ? ct / p.Wh : 0, jc = has_new ? ct - nr * p.Wh : 0;
-        const uint32_t src_nr = 2u * static_cast<uint32_t>(nr) * static_cast<uint32_t>(p.f_rowbytes);
-        uint32_t coff[4];
-        const uint32_t cok = f32_s2d_offsets(p, jc, coff);
+        // this thread's pixels of a continuation tile (Rt new rows: tile_px <= 256, so at most
+        // two per thread): new row nr, column jc, source offsets
+        constexpr int kMaxNew = 2;
+        int nr[kMaxNew], jc[kMaxNew];
+        uint32_t src_nr[kMaxNew], coff[kMaxNew][4], cok[kMaxNew];
+#pragma unroll
+        for (int u = 0; u < kMaxNew; ++u) {
+            const int px = ct + u * kNumCvtWarps * 32;
+            const int pq = px < tile_px ? px : 0;
+            nr[u] = pq / p.Wh;
+            jc[u] = pq - nr[u] * p.Wh;
+            src_nr[u] = 2u * static_cast<uint32_t>(nr[u]) * static_cast<uint32_t>(p.f_rowbytes);
+            cok[u] = f32_s2d_offsets(p, jc[u], coff[u]);
+        }
         named_bar_sync(2, kNumCvtWarps * 32);           // the zero area is written
         int base = 0;                                    // ring row of the tile's halo row 0
         int g = 0;
@@ -433,14 +525,17 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             if (cont) {
                 base += p.Rt;
                 if (base >= NR) base -= NR;
-                if (has_new) {          // halo row HR - Rt + nr from staged rows 2 nr, 2 nr + 1
-                    int slot = base + p.HR - p.Rt + nr;
+#pragma unroll
+                for (int u = 0; u < kMaxNew; ++u) {
+                    if (ct + u * kNumCvtWarps * 32 >= tile_px) break;
+                    // halo row HR - Rt + nr from staged rows 2 nr, 2 nr + 1
+                    int slot = base + p.HR - p.Rt + nr[u];
                     if (slot >= NR) slot -= NR;
                     uint32_t addr[4], w[4];
-                    f32_s2d_addr(src + src_nr, coff, cok, zero, addr);
+                    f32_s2d_addr(src + src_nr[u], coff[u], cok[u], zero, addr);
                     if (p.f_c == 3) f32_s2d_pixel<3>(p, addr, w);
                     else f32_s2d_pixel<4>(p, addr, w);
-                    const uint32_t dst = ring + static_cast<uint32_t>(slot) * rowpx + 16u * static_cast<uint32_t>(jc);
+                    const uint32_t dst = ring + static_cast<uint32_t>(slot) * rowpx + 16u * static_cast<uint32_t>(jc[u]);
                     sts128(dst, w[0], w[1], w[2], w[3]);
                     sts128(dst + mirror, w[0], w[1], w[2], w[3]);
                 }

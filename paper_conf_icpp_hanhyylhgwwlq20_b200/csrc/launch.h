@@ -22,7 +22,7 @@ cudaError_t launch_fwd(const Launch &L, bool is4, int out, bool zx, const CUtens
 cudaError_t launch_fwd2(const Launch &L, bool is4, int out, const CUtensorMap &xm, const CUtensorMap &wm,
                         const CUtensorMap &ym, const ConvParams &p);
 cudaError_t launch_halo(const Launch &L, bool is4, int out, const CUtensorMap &hm, const CUtensorMap &bm,
-                        const CUtensorMap &ym, const ConvParams &p);
+                        const CUtensorMap &ym, const ConvParams &p, bool cm = false);
 cudaError_t launch_trans(const Launch &L, bool is4, int out, bool m64, const CUtensorMap &xm,
                          const CUtensorMap &wm, const CUtensorMap &ym, const ConvParams &p);
 

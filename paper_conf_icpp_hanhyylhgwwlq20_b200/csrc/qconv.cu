@@ -643,9 +643,12 @@ bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, bool ch
 // ------------------------------------------------------------------ halo mode (stride 1)
 // f32_row_bytes > 0: the fused fp32-quantization stem (halo.cuh F32): the staging ring holds
 // the tile's 2*HR fp32 input rows of f32_row_bytes each instead of packed codes.
-bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f32_row_bytes = 0) {
+// cm: the channel-major variant (halo.cuh CM): K = 64 output channels on TMEM lanes, N = Rt
+// padded rows of Wh = round_up(W + 2 pad, 8) pixels (<= 256), the channel-pair epilogue.
+bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f32_row_bytes = 0, bool cm = false) {
     if (d->stride_h != 1 || d->stride_w != 1 || d->dil_h != 1 || d->dil_w != 1) return false;
     if (d->x_zero != 0 || !is_packed_out(d->y_t)) return false;
+    if (cm && (d->k != 64 || d->rounding == QC_ROUND_TFLITE)) return false;
     const bool is4 = g.bits == 4;
     const int C8 = d->c;                                 // int8 bytes per pixel after widening
     const bool tap_pair = !is4 && C8 == 16;
@@ -654,12 +657,13 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f
     } else if (C8 % 32) {
         return false;
     }
-    const int Wh = d->w + 2 * d->pad_w;
-    if (Wh > qc::kBM || Wh > 256) return false;
+    const int Wh = cm ? (d->w + 2 * d->pad_w + 7) / 8 * 8 : d->w + 2 * d->pad_w;
+    const int tile_px = cm ? 256 : qc::kBM;               // accumulator rows (pixels) per tile
+    if (Wh > tile_px || Wh > 256) return false;
     if (d->r * d->s == 1) return false;                 // no tap reuse: the im2col GEMM path is better
-    const int Rt = qc::kBM / Wh;
+    const int Rt = tile_px / Wh;
     const int tpi = (g.P + Rt - 1) / Rt;
-    if (static_cast<double>(g.P) * g.Q / (static_cast<double>(tpi) * qc::kBM) < 0.7) return false;
+    if (static_cast<double>(g.P) * g.Q / (static_cast<double>(tpi) * tile_px) < 0.7) return false;
     const int HR = Rt + d->r - 1;
     const int nplanes = C8 / 16;
     const int nch = g.c_bytes / 16;                      // TMA channel chunks (packed for 4-bit)
@@ -675,6 +679,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f
     const int ybits = dtype_bits(d->y_t);
     const int tile_row_bytes = BN * ybits / 8;
     const int y_gw = tile_row_bytes >= 128 ? 128 : tile_row_bytes;
+    const int ystg_rows = cm ? 256 : 128;
     if (!((static_cast<int64_t>(d->k) * ybits / 8) % 16 == 0 &&
           (y_gw == 32 || y_gw == 64 || (y_gw == 128 && tile_row_bytes % 128 == 0))))
         return false;
@@ -685,8 +690,8 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f
     const uint32_t plane = static_cast<uint32_t>(HR * Wh * 16);
     // the fused fp32 stem keeps one ring of HR + Rt code rows, each stored twice, plus a
     // 64-byte zero area (halo.cuh F32) instead of a code halo per stage
-    const uint32_t ringb = f32_row_bytes ? static_cast<uint32_t>(align_up(static_cast<size_t>(2 * (HR + Rt)) * Wh * 16 + 64, 1024)) : 0u;
-    const uint32_t hx = f32_row_bytes ? 0u : static_cast<uint32_t>(align_up(static_cast<size_t>(nplanes) * plane, 1024));
+    const uint32_t ringb = f32_row_bytes ? static_cast<uint32_t>(align_up(static_cast<size_t>(2 * (HR + Rt)) * Wh * 16 + 64 + (cm ? 256 : 0), 1024)) : 0u;
+    const uint32_t hx = f32_row_bytes ? 0u : static_cast<uint32_t>(align_up(static_cast<size_t>(nplanes) * plane + (cm ? 256 : 0), 1024));
     const uint32_t hp = f32_row_bytes ? static_cast<uint32_t>(align_up(static_cast<size_t>(2 * HR) * f32_row_bytes, 1024))
                         : (is4 ? static_cast<uint32_t>(align_up(static_cast<size_t>(nch) * plane, 1024)) : 0u);
     const uint32_t bres = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * KG8, 1024));
@@ -694,7 +699,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f
     int n_ystg = QC_MAX_YSTG;
     uint32_t ystg = 0, fixed = 0;
     for (;; --n_ystg) {
-        ystg = static_cast<uint32_t>(n_ystg) * 128u * static_cast<uint32_t>(tile_row_bytes);
+        ystg = static_cast<uint32_t>(n_ystg) * static_cast<uint32_t>(ystg_rows) * static_cast<uint32_t>(tile_row_bytes);
         fixed = bres + ringb + ystg + static_cast<uint32_t>(qc::kMaxBN) * 16u + 128u + 2048u +
                 8u * static_cast<uint32_t>(d->r * d->s * nplanes);
         if (n_ystg == 2 || fixed + 3 * (hx + hp) <= 227u * 1024u) break;
@@ -740,8 +745,11 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f
     const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 5 + 2 * qc::kMaxYstg + 1) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
     if (pl->smem_bytes > 227u * 1024u) return false;
-    p.idesc = qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), act_signed(d), dtype_signed(d->w_t));
-    pl->tmem_cols = pow2_cols(2 * BN);
+    // kind::i8 takes N = 8 or a multiple of 16: the padded columns read halo pixels past the
+    // tile (slack below) into accumulator columns nobody stores
+    p.idesc = cm ? qc::make_idesc_i8(64u, static_cast<uint32_t>((Rt * Wh + 15) / 16 * 16), dtype_signed(d->w_t), act_signed(d))
+                 : qc::make_idesc_i8(qc::kBM, static_cast<uint32_t>(BN), act_signed(d), dtype_signed(d->w_t));
+    pl->tmem_cols = cm ? 512u : pow2_cols(2 * BN);
     p.tmem_cols = pl->tmem_cols;
     p.y_zero = d->y_zero; p.clamp_lo = d->clamp_lo; p.clamp_hi = d->clamp_hi; p.x_zero = 0;
     p.need_clamp = (d->clamp_lo > dtype_min(d->y_t) || d->clamp_hi < dtype_max(d->y_t)) ? 1 : 0;
@@ -749,11 +757,12 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f
     const int sms = num_sms();
     int grid = std::min<int64_t>(num_tiles, sms / n_tiles_n * n_tiles_n);
     grid = std::max(grid / n_tiles_n * n_tiles_n, n_tiles_n);
-    pl->kernel = QC_KERNEL_HALO;
+    pl->kernel = cm ? QC_KERNEL_HALO_T : QC_KERNEL_HALO;
     pl->grid = grid;
-    pl->threads = (is4 || f32_row_bytes) ? 512 : 384;
+    pl->threads = cm ? ((is4 || f32_row_bytes) ? qc::kTThreads4 : qc::kTThreads8)
+                     : ((is4 || f32_row_bytes) ? 512 : 384);
     pl->BN = BN;
-    pl->BM = qc::kBM;
+    pl->BM = cm ? Rt * Wh : qc::kBM;
     pl->n_tiles_n = n_tiles_n;
     pl->num_tiles = static_cast<int>(num_tiles);
     pl->stages = stages;
@@ -762,7 +771,7 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f
 
 qc_status encode_halo_maps(const qconv_desc *d, const Geometry &g, const qc::ConvParams &p,
                            const void *x, const void *w8, void *y, CUtensorMap *hm, CUtensorMap *bm,
-                           CUtensorMap *ym) {
+                           CUtensorMap *ym, bool cm = false) {
     const Driver &drv = driver();
     if (!drv.tiled) return cuda_fail(drv.err);
     const cuuint64_t cb = static_cast<cuuint64_t>(g.c_bytes);
@@ -790,7 +799,18 @@ qc_status encode_halo_maps(const qconv_desc *d, const Geometry &g, const qc::Con
         if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
         small_tensor_fixup(hm, static_cast<uint64_t>(g.x_bytes));
     }
-    {   // weights: [K-chunk][k][16 B] view of int8 KRSC
+    if (cm) {   // weights: [K-chunk][k / 16][h][i][16 B] view, smem row 16 g + 8 h + i = channel 16 g + 2 i + h
+        const cuuint64_t kg = static_cast<cuuint64_t>(d->r) * d->s * d->c;
+        cuuint64_t dims[5] = {16, 8, 2, static_cast<cuuint64_t>(d->k / 16), kg / 16};
+        cuuint64_t strides[4] = {2 * kg, kg, 16 * kg, 16};
+        cuuint32_t box[5] = {16, 8, 2, static_cast<cuuint32_t>(p.BN / 16), static_cast<cuuint32_t>(kg / 16)};
+        cuuint32_t es[5] = {1, 1, 1, 1, 1};
+        CUresult r = drv.tiled(bm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 5, const_cast<void *>(w8), dims, strides,
+                               box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return cuda_fail(cudaErrorInvalidValue);
+        small_tensor_fixup(bm, static_cast<uint64_t>(g.w8_bytes));
+    } else {   // weights: [K-chunk][k][16 B] view of int8 KRSC
         const cuuint64_t kg = static_cast<cuuint64_t>(d->r) * d->s * d->c;
         cuuint64_t dims[3] = {16, static_cast<cuuint64_t>(d->k), kg / 16};
         cuuint64_t strides[2] = {kg, 16};
@@ -809,7 +829,7 @@ qc_status encode_halo_maps(const qconv_desc *d, const Geometry &g, const qc::Con
                               static_cast<cuuint64_t>(d->n)};
         cuuint64_t strides[3] = {row, row * g.Q, row * g.Q * g.P};
         cuuint32_t box[4] = {static_cast<cuuint32_t>(p.y_gw), static_cast<cuuint32_t>(g.Q),
-                             static_cast<cuuint32_t>(p.Rt), 1};
+                             static_cast<cuuint32_t>(cm ? 1 : p.Rt), 1};
         cuuint32_t es[4] = {1, 1, 1, 1};
         CUresult r = drv.tiled(ym, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, y, dims, strides, box, es,
                                CU_TENSOR_MAP_INTERLEAVE_NONE, swizzle_for(p.y_gw),
@@ -915,12 +935,13 @@ struct Choice {
 };
 
 // Resolve a choice to a plan on the exec descriptor; AUTO = the default rule
-// (halo -> channel-major -> CTA pair -> im2col).
+// (channel-major halo -> halo -> channel-major 1x1 -> CTA pair -> im2col).
 bool resolve(const Exec &ex, Choice c, Plan *pl) {
     const qconv_desc *e = &ex.e;
     const Geometry &g = ex.g;
     const bool special_ok = !needs_general_only(ex);       // halo / channel / pair eligibility
     if (c.kernel == QC_KERNEL_AUTO) {
+        if (special_ok && make_halo_plan(e, g, pl, 0, true)) return true;   // K = 64: channel-major halo
         if (special_ok && make_halo_plan(e, g, pl)) return true;
         if (special_ok && make_trans_plan(e, g, 0, false, pl)) return true;
         Plan p1;
@@ -932,6 +953,9 @@ bool resolve(const Exec &ex, Choice c, Plan *pl) {
     switch (c.kernel) {
         case QC_KERNEL_HALO:
             if (!special_ok || !make_halo_plan(e, g, pl)) return false;
+            return c.bn == 0 || c.bn == pl->BN;
+        case QC_KERNEL_HALO_T:
+            if (!special_ok || !make_halo_plan(e, g, pl, 0, true)) return false;
             return c.bn == 0 || c.bn == pl->BN;
         case QC_KERNEL_CHANNEL:
             return special_ok && make_trans_plan(e, g, c.bn, true, pl);
@@ -961,6 +985,7 @@ std::vector<Choice> candidates(const Exec &ex) {
         }
     };
     try_add(QC_KERNEL_HALO, 0);
+    try_add(QC_KERNEL_HALO_T, 0);
     try_add(QC_KERNEL_CHANNEL, 64);
     try_add(QC_KERNEL_CHANNEL, 128);
     const int kmax = std::min(qc::kMaxBN, (ex.e.k + 15) / 16 * 16);
@@ -1004,7 +1029,8 @@ void fill_plan_out(const Exec &ex, const Plan &pl, qconv_plan *o) {
     o->threads = pl.threads;
     o->num_tiles = pl.num_tiles;
     o->smem_bytes = static_cast<int32_t>(pl.smem_bytes);
-    o->tmem_cols = static_cast<int32_t>(pl.kernel == QC_KERNEL_HALO || pl.kernel == QC_KERNEL_CHANNEL
+    o->tmem_cols = static_cast<int32_t>(pl.kernel == QC_KERNEL_HALO || pl.kernel == QC_KERNEL_HALO_T ||
+                                                pl.kernel == QC_KERNEL_CHANNEL
                                             ? pl.cp.tmem_cols : pl.tmem_cols);
     o->prologue = ex.prologue;
     o->epilogue_mode = (needs_general_only(ex) || ex.e.rounding == QC_ROUND_TFLITE) ? 2 : -1;
@@ -1139,10 +1165,13 @@ qc_status launch_plan(const Exec &ex, Plan &pl, const void *x, const void *w8, c
     std::memset(&m2, 0, sizeof(m2));
     switch (pl.kernel) {
         case QC_KERNEL_HALO:
-            s = encode_halo_maps(e, g, p, x, w8, y, &m0, &m1, &m2);
+        case QC_KERNEL_HALO_T: {
+            const bool cm = pl.kernel == QC_KERNEL_HALO_T;
+            s = encode_halo_maps(e, g, p, x, w8, y, &m0, &m1, &m2, cm);
             if (s != QC_OK) return s;
-            err = qc::launch_halo(L, is4, out, m0, m1, m2, p);
+            err = qc::launch_halo(L, is4, out, m0, m1, m2, p, cm);
             break;
+        }
         case QC_KERNEL_CHANNEL:
             p.stg_sw = is4 ? packed_sw_mask(pl.bkp) : 0;
             s = encode_x_map(e, g, x, pl.bkp, is4 ? packed_swizzle(pl.bkp) : swizzle_for(pl.BK), &m0, p.Wh);
@@ -1253,7 +1282,13 @@ qc_status derive_qexec(const qconv_desc *d, qc_ftype xt, QExec *qx) {
             ex.off_w = ex.off_x = ex.off_zx = ex.off_cs = ex.off_x1 = 0;
             ex.prologue = ex.wprep_needed ? 1 : 0;
             ex.ws_total = ex.wprep_needed ? align_up(ex.prep_bytes, 256) : 0;
-            if (make_halo_plan(&ex.e, ex.g, &qx->pl, static_cast<uint32_t>(d->w) * d->c * 4u)) {
+            // the fused stem runs the channel-major halo when it is eligible (K = 64), unless a
+            // plan choice for `d` asks for the pixel-major one
+            const uint32_t frow = static_cast<uint32_t>(d->w) * d->c * 4u;
+            const Choice c = current_choice(d);
+            const bool cm_first = c.kernel != QC_KERNEL_HALO;
+            if ((cm_first && make_halo_plan(&ex.e, ex.g, &qx->pl, frow, true)) ||
+                (c.kernel != QC_KERNEL_HALO_T && make_halo_plan(&ex.e, ex.g, &qx->pl, frow, false))) {
                 qx->fused = true;
                 qx->ws_total = ex.ws_total;
                 return QC_OK;
@@ -1304,7 +1339,8 @@ qc_status launch_fused_stem(QExec &qx, const void *x, float in_scale, const void
     p.fd_s = qc::make_fastdiv(static_cast<uint32_t>(std::max(1, p.S)));
     p.fd_tpi = qc::make_fastdiv(static_cast<uint32_t>(std::max(1, p.tiles_per_img)));
     alignas(64) CUtensorMap hm, bm, ym;
-    qc_status s = encode_halo_maps(e, ex.g, p, x, w8, y, &hm, &bm, &ym);
+    const bool cm = pl.kernel == QC_KERNEL_HALO_T;
+    qc_status s = encode_halo_maps(e, ex.g, p, x, w8, y, &hm, &bm, &ym, cm);
     if (s != QC_OK) return s;
     {   // fp32 input rows as raw 8-byte elements: [n][h][k pieces][row/k]; each row piece is one
         // long contiguous TMA row (a 16-byte inner box would cost one request per 16 bytes);
@@ -1332,7 +1368,7 @@ qc_status launch_fused_stem(QExec &qx, const void *x, float in_scale, const void
     static const bool no_pdl = std::getenv("QC_NO_PDL") != nullptr;
     L.pdl = !no_pdl;
     debug_attach(p, st);
-    cudaError_t err = qc::launch_halo(L, false, out_kind(e->y_t), hm, bm, ym, p);
+    cudaError_t err = qc::launch_halo(L, false, out_kind(e->y_t), hm, bm, ym, p, cm);
     if (err != cudaSuccess) return cuda_fail(err);
     debug_dump(p, st);
     return QC_OK;
@@ -1548,7 +1584,8 @@ qc_status qconv_debug_plan(const qconv_desc *d, qconv_plan *out) {
 
 qc_status qconv_plan_set(const qconv_desc *d, const qconv_plan *choice) {
     Exec ex;
-    qc_status s = derive_exec(d, true, &ex);
+    qconv_desc tmp;          // 4-bit odd-C stems: validated on their byte-code view (the fused path)
+    qc_status s = derive_exec_for_weights(d, &ex, &tmp);
     if (s != QC_OK) return s;
     const std::string key = desc_key(d);
     std::lock_guard<std::mutex> lk(g_plan_mu);

@@ -53,7 +53,7 @@ def trunk256(request):
 def test_trunk256_plans_cover_the_wide_tiles(trunk256):
     plans = [(L["plan"]["kernel_name"], L["plan"]["bn"]) for L in trunk256.layers]
     assert ("pair", 256) in plans
-    assert {"halo", "channel"} <= {k for k, _ in plans}
+    assert {"halo_t", "channel"} <= {k for k, _ in plans}
 
 
 def test_trunk256_chain_vs_oracle(trunk256):

@@ -83,6 +83,7 @@ def _assert_same(got, ref, what=""):
 # one shape per kernel family, with the family forced through the plan API
 FAMILY_SHAPES = {
     "halo": (ConvShape("halo", 2, 14, 14, 64, 128, 3, 3, 1, 1), qc.QC_KERNEL_HALO, 0),
+    "halo_t": (ConvShape("halo_t", 2, 14, 14, 64, 64, 3, 3, 1, 1), qc.QC_KERNEL_HALO_T, 0),
     "channel": (ConvShape("chan", 2, 10, 12, 64, 128, 1, 1), qc.QC_KERNEL_CHANNEL, 128),
     "pair": (ConvShape("pair", 2, 9, 9, 64, 128, 3, 3, 1, 1), qc.QC_KERNEL_PAIR, 128),
     "im2col": (ConvShape("im2col", 2, 11, 9, 64, 128, 3, 3, 2, 1), qc.QC_KERNEL_IM2COL, 128),
@@ -117,7 +118,9 @@ def test_requant_full_domain_every_kernel(family, bits, out):
     li = make_layer_inputs(cs, bits, seed=zlib.crc32(f"{family}{bits}{out}".encode()) % 997,
                            relu=out.startswith("u"), signed_out=out.startswith("s"))
     rng = np.random.default_rng(zlib.crc32(family.encode()) + bits)
-    m, n = _requant_domain(cs.k, rng)
+    m, n = _requant_domain(max(cs.k, 128), rng)
+    if cs.k < 128:      # K = 64 (channel-major halo): every other channel keeps all four chunk kinds
+        m, n = m[::128 // cs.k].copy(), n[::128 // cs.k].copy()
     ref = oracle.conv2d_layer(li, mult=m, shift=n)
     got, plan = _gpu(li, m, n, kernel=kern, bn=bn)
     assert plan["kernel"] == kern
@@ -143,10 +146,10 @@ def test_requant_mid_hole_worked_example():
 @pytest.mark.parametrize("family", list(FAMILY_SHAPES))
 @pytest.mark.parametrize("bits", [8, 4])
 def test_tflite_rounding_every_kernel(family, bits):
-    """TFLite rounding on every kernel that takes it (the channel-major kernel does not: its
-    epilogue would spill registers; its 1x1 layers then run on the im2col kernel)."""
+    """TFLite rounding on every kernel that takes it (the channel-major kernels do not: their
+    epilogue would spill registers; such layers then run on another kernel, by the default rule)."""
     cs, kern, bn = FAMILY_SHAPES[family]
-    if family == "channel":
+    if family in ("channel", "halo_t"):
         kern, bn = None, 0
     li = make_layer_inputs(cs, bits, seed=5 + bits, relu=False, signed_out=True)
     rng = np.random.default_rng(7 + bits)
@@ -334,8 +337,9 @@ def test_autotune_records_an_exact_plan():
 
 
 @pytest.mark.parametrize("bits", [8, 4])
-@pytest.mark.parametrize("n_img,relu", [(2, True), (1, False)])
-def test_forward_quantize_fused_stem(bits, n_img, relu):
+@pytest.mark.parametrize("n_img,relu", [(2, True), (1, False), (5, True)])
+@pytest.mark.parametrize("kernel", ["halo_t", "halo"])
+def test_forward_quantize_fused_stem(bits, n_img, relu, kernel):
     """qconv2d_forward_quantize on the C = 3 stem: one kernel quantizes the fp32 rows (Z4) into
     its space-to-depth operand tile; compared with oracle quantize (+ a zero-point channel) then
     the oracle's direct 7x7/s2 conv.  Inputs include NaN, +-inf and exact quantization ties."""
@@ -353,15 +357,21 @@ def test_forward_quantize_fused_stem(bits, n_img, relu):
                      clamp_lo=li.clamp_lo, clamp_hi=li.clamp_hi)
     w = torch.from_numpy(np.ascontiguousarray(pack_codes(li.w_codes[..., :3], S8))).to(DEV)
     b, mm, nn = (torch.from_numpy(a).to(DEV) for a in (li.bias, m, n))
-    y = qc.qconv2d_forward_quantize(d, torch.from_numpy(xf).to(DEV), s_x, w, b, mm, nn)
-    torch.cuda.synchronize()
-    _assert_same(y.cpu().numpy(), ref, "fused stem (unprepared weights)")
-    wp = qc.qconv_prepare_weights(d, w)
-    d.w_prepared = 1
-    assert qc._lib().qconv2d_quantize_workspace_size(d, qc.QC_F32) == 0     # one kernel, no workspace
-    y = qc.qconv2d_forward_quantize(d, torch.from_numpy(xf).to(DEV), s_x, wp, b, mm, nn)
-    torch.cuda.synchronize()
-    _assert_same(y.cpu().numpy(), ref, "fused stem (prepared weights)")
+    want = qc.QC_KERNEL_HALO_T if kernel == "halo_t" else qc.QC_KERNEL_HALO
+    try:
+        for prepared in (False, True):
+            if prepared:
+                w = qc.qconv_prepare_weights(d, w)
+                d.w_prepared = 1
+                assert qc._lib().qconv2d_quantize_workspace_size(d, qc.QC_F32) == 0   # one kernel
+            if kernel == "halo":        # the pixel-major halo, chosen through the plan API
+                qc.qconv_plan_set(d, qc.QC_KERNEL_HALO, 0)
+            assert qc.qconv_debug_plan_quantize(d)["kernel"] == want
+            y = qc.qconv2d_forward_quantize(d, torch.from_numpy(xf).to(DEV), s_x, w, b, mm, nn)
+            torch.cuda.synchronize()
+            _assert_same(y.cpu().numpy(), ref, f"fused stem {kernel} (prepared={prepared})")
+    finally:
+        qc.qconv_plan_clear()
 
 
 @pytest.mark.parametrize("cs,bits,x_zero,bf16", [
