@@ -127,13 +127,17 @@ def test_plans_on_the_host():
         qc.qconv_plan_set(d, qc.QC_KERNEL_CHANNEL, 128)                      # 3x3: ineligible
     qc.qconv_plan_set(d, None)
     assert qc.qconv_debug_plan(d)["kernel_name"] == "pair"
-    # 1x1 -> channel-major; stem in s2d form -> halo; int32 output -> im2col
+    # 1x1 -> channel-major; stem in s2d form (K = 64) -> channel-major halo; int32 output -> im2col
     d1 = qc.make_desc(32, 56, 56, 64, 256, 1, 1, x_t=qc.QC_U4, w_t=qc.QC_S4, y_t=qc.QC_S4,
                       w_prepared=1)
     assert qc.qconv_debug_plan(d1)["kernel_name"] == "channel"
     stem = qc.make_desc(8, 224, 224, 3, 64, 7, 7, stride=2, pad=3, w_prepared=1)
     ps = qc.qconv_debug_plan(stem)
-    assert ps["kernel_name"] == "halo" and ps["prologue"] == 2
+    assert ps["kernel_name"] == "halo_t" and ps["prologue"] == 2
+    assert ps["threads"] == 640 and ps["tmem_cols"] == 512 and ps["bm"] == 240   # 2 rows of 120 pixels
+    qc.qconv_plan_set(stem, qc.QC_KERNEL_HALO, 0)                                 # the pixel-major one
+    assert qc.qconv_debug_plan(stem)["kernel_name"] == "halo"
+    qc.qconv_plan_set(stem, None)
     d32 = qc.make_desc(2, 9, 9, 64, 48, 3, 3, pad=1, y_t=qc.QC_S32)
     assert qc.qconv_debug_plan(d32)["kernel_name"] == "im2col"
 
