@@ -382,11 +382,17 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             tc_fence_after();
             if (ew == 0 && lane == 0) trace_ev(p, 5, it);
             mbar_wait(&sfree[sb], sphase ^ 1u);
+            if (ew == 0 && lane == 0) trace_ev(p, 10, it);
             const uint32_t ystg = ystg_base + static_cast<uint32_t>(sb) * p.ystg_bytes;
             uint32_t va[32];
             tmem_ld_16x256b_x8(taddr0 + static_cast<uint32_t>(buf * 256), va);
+            // the multipliers re-enter the loop as plain 32-bit registers: hoisted out of it as
+            // sign-extended 64-bit values they turned every product into a 64x64 multiply
+            asm volatile("" : "+r"(ce.m), "+r"(co.m));
             tmem_wait_ld_regs(va);
+            if (ew == 0 && lane == 0) trace_ev(p, 13, it);
             t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, va, ystg, row0, boff);
+            if (ew == 0 && lane == 0) trace_ev(p, 14, it);
             tc_fence_before();
             fence_proxy_async_smem();                 // staging writes -> visible to the TMA store
             __syncwarp();
@@ -525,19 +531,26 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             if (cont) {
                 base += p.Rt;
                 if (base >= NR) base -= NR;
+                // both pixels computed unconditionally (a thread without a second pixel redoes
+                // its first), so the 2 x 12 load -> quantize chains interleave; stores predicated
+                uint32_t w[kMaxNew][4];
 #pragma unroll
                 for (int u = 0; u < kMaxNew; ++u) {
-                    if (ct + u * kNumCvtWarps * 32 >= tile_px) break;
-                    // halo row HR - Rt + nr from staged rows 2 nr, 2 nr + 1
-                    int slot = base + p.HR - p.Rt + nr[u];
-                    if (slot >= NR) slot -= NR;
-                    uint32_t addr[4], w[4];
+                    uint32_t addr[4];
                     f32_s2d_addr(src + src_nr[u], coff[u], cok[u], zero, addr);
-                    if (p.f_c == 3) f32_s2d_pixel<3>(p, addr, w);
-                    else f32_s2d_pixel<4>(p, addr, w);
-                    const uint32_t dst = ring + static_cast<uint32_t>(slot) * rowpx + 16u * static_cast<uint32_t>(jc[u]);
-                    sts128(dst, w[0], w[1], w[2], w[3]);
-                    sts128(dst + mirror, w[0], w[1], w[2], w[3]);
+                    if (p.f_c == 3) f32_s2d_pixel<3>(p, addr, w[u]);
+                    else f32_s2d_pixel<4>(p, addr, w[u]);
+                }
+#pragma unroll
+                for (int u = 0; u < kMaxNew; ++u) {
+                    if (ct + u * kNumCvtWarps * 32 < tile_px) {
+                        // halo row HR - Rt + nr from staged rows 2 nr, 2 nr + 1
+                        int slot = base + p.HR - p.Rt + nr[u];
+                        if (slot >= NR) slot -= NR;
+                        const uint32_t dst = ring + static_cast<uint32_t>(slot) * rowpx + 16u * static_cast<uint32_t>(jc[u]);
+                        sts128(dst, w[u][0], w[u][1], w[u][2], w[u][3]);
+                        sts128(dst + mirror, w[u][0], w[u][1], w[u][2], w[u][3]);
+                    }
                 }
             } else {
                 base = 0;

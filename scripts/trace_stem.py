@@ -34,7 +34,7 @@ t = np.fromfile(out, dtype=np.uint64).reshape(-1, 16, 1024).astype(np.int64)[-1]
 t0 = min(v for v in t.reshape(-1) if v > 0)
 names = {0: "prod", 2: "mma_acc_free", 3: "mma_in", 1: "mma_fenced", 11: "mma_issued", 12: "commit_empty",
          4: "commit_tfull", 5: "epi_acc_full", 6: "epi_done", 7: "store", 8: "cvt_in", 10: "epi_stg_free", 13: "epi_ld_done", 14: "epi_requant_done", 9: "cvt_done"}
-if L["plan"]["kernel_name"] != "halo":
+if L["plan"]["kernel_name"] not in ("halo", "halo_t"):
     names = {i: f"ev{i}" for i in range(16)}
 for ev, nm in names.items():
     row = t[ev][t[ev] > 0] - t0
