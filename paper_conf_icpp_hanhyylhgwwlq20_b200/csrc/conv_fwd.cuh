@@ -159,7 +159,20 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                     tc_fence_after();
                     const uint32_t a_addr = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
                     const uint32_t b_addr = smem_u32(smem + p.off_b + stage * p.b_stage_bytes);
-                    if (p.pair) {
+                    if (IS4 && p.a_tmem_col > 0) {
+                        // widened A rows in TMEM (converter warps), B from shared memory
+                        const uint64_t bd0 = make_smem_desc(b_addr, 16u, sbo, p.sw_layout);
+                        const uint32_t blo = static_cast<uint32_t>(bd0), bhi = static_cast<uint32_t>(bd0 >> 32);
+                        const uint32_t a_t = tmem_base + static_cast<uint32_t>(p.a_tmem_col + stage * (p.BK / 4));
+                        if (ksteps == 4) {
+#pragma unroll
+                            for (int k = 0; k < 4; ++k)
+                                mma_i8_ts_warp(d_tmem, a_t + 8u * k, blo + 2u * k, bhi, p.idesc, (kb | k) != 0 ? 1u : 0u);
+                        } else {
+                            for (int k = 0; k < ksteps; ++k)
+                                mma_i8_ts_warp(d_tmem, a_t + 8u * k, blo + 2u * k, bhi, p.idesc, (kb | k) != 0 ? 1u : 0u);
+                        }
+                    } else if (p.pair) {
                         // canonical no-swizzle K-major: core matrices 8 rows x 16 B; the two
                         // 16-byte K halves (filter taps) are LBO apart, 8-row groups SBO = 128 B
                         const uint64_t ad = make_smem_desc(a_addr, kBM * 16u, 128u, 0u);
@@ -322,8 +335,40 @@ qconv_fwd_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant
                 mbar_wait(&full[stage], phase);
                 if (ct == 0) trace_ev(p, 8, cstage++);
                 const uint32_t stg = smem_u32(smem + p.off_stg + stage * p.stg_stage_bytes);
-                const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
-                widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
+                if (p.a_tmem_col > 0) {
+                    // thread = accumulator row m = ct: its pixel's bkp packed bytes -> 2 bkp widened
+                    // bytes (chunk q: lo words then hi words, the order widen_stage writes) ->
+                    // TMEM lane m, columns a_tmem_col + stage BK/4 ..  The packed staging is
+                    // TMA-swizzled (16-byte chunk index ^= address bits 7+): conflict-free rows.
+                    uint32_t o[32];
+                    const uint32_t ssw = static_cast<uint32_t>(p.stg_sw);
+                    const uint32_t rowoff = static_cast<uint32_t>(ct) * static_cast<uint32_t>(p.bkp);
+                    // all four loads first (a short row reads past its end into the next row /
+                    // stage, unused), then the widening: one latency, not four
+                    uint4 v[4];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        const uint32_t so = rowoff + 16u * q;
+                        v[q] = lds128u(stg + (so ^ (((so >> 7) & ssw) << 4)));
+                    }
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        widen_word(v[q].x, xo, o[8 * q + 0], o[8 * q + 4]);
+                        widen_word(v[q].y, xo, o[8 * q + 1], o[8 * q + 5]);
+                        widen_word(v[q].z, xo, o[8 * q + 2], o[8 * q + 6]);
+                        widen_word(v[q].w, xo, o[8 * q + 3], o[8 * q + 7]);
+                    }
+                    const uint32_t ta = tmem_base + (static_cast<uint32_t>((warp & 3) * 32) << 16) +
+                                        static_cast<uint32_t>(p.a_tmem_col + stage * (p.BK / 4));
+                    if (p.bkp == 64) tmem_st_32x32b_x32(ta, o);
+                    else if (p.bkp == 32) tmem_st_32x32b_x16(ta, o);
+                    else tmem_st_32x32b_x8(ta, o);
+                    tmem_wait_st();
+                    tc_fence_before();
+                } else {
+                    const uint32_t adst = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
+                    widen_stage(stg, adst, ct, nchunks, cshift, bkb, sw, xo, static_cast<uint32_t>(p.stg_sw));
+                }
                 fence_proxy_async_smem();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&aready[stage]);

@@ -398,6 +398,12 @@ bool needs_general_only(const Exec &ex) {
     return ex.zx || ex.zw || !is_packed_out(ex.e.y_t);
 }
 
+#ifdef QC_NO_A_TMEM          // build-time A/B switch (same bytes): widened A tiles in shared memory
+constexpr bool g_no_a_tmem = true;
+#else
+constexpr bool g_no_a_tmem = false;
+#endif
+
 // im2col kernel (conv_fwd.cuh).  bn_req = 0: the default N tile (largest <= 256, halved
 // while the grid would not fill the GPU -- P:L321: at small batch the tiling decides how
 // well the machine is filled).
@@ -425,7 +431,13 @@ bool make_plan(const qconv_desc *d, const Geometry &g, int bn_req, Plan *pl) {
     pl->n_tiles_n = (d->k + BN - 1) / BN;
     pl->num_tiles = m_tiles * pl->n_tiles_n;
     pl->tmem_cols = pow2_cols(2 * BN);
-    const uint32_t a_bytes = static_cast<uint32_t>(qc::kBM * pl->BK);
+    // 4-bit: the widened A tile can live in TMEM (conv_fwd.cuh): one BK/4-column slab per stage
+    // after the two accumulators -- no widened copy in shared memory and no A operand reads of
+    // it, but the 512 columns cap the ring depth
+    const int a_cols = pl->BK / 4;
+    const int tmem_stages = is4 && !pair && !g_no_a_tmem ? (512 - 2 * BN) / a_cols : 0;
+    const bool a_tmem = tmem_stages >= 4;
+    const uint32_t a_bytes = a_tmem ? 0u : static_cast<uint32_t>(qc::kBM * pl->BK);
     const uint32_t b_bytes = static_cast<uint32_t>(align_up(static_cast<size_t>(BN) * pl->BK, 1024));
     const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(qc::kBM * pl->bkp) : 0u;
     const uint32_t per_stage = a_bytes + b_bytes + stg_bytes;
@@ -441,10 +453,13 @@ bool make_plan(const qconv_desc *d, const Geometry &g, int bn_req, Plan *pl) {
     const uint32_t budget = 227u * 1024u - 1024u - fixed;
     int stages = static_cast<int>(budget / per_stage);
     stages = std::min(stages, 32);     // deep rings: TMA latency is ~1-3 us under load
+    if (a_tmem) stages = std::min(stages, tmem_stages);
     if (stages < 2) return false;
     pl->stages = stages;
+    if (a_tmem) pl->tmem_cols = 512;
     qc::ConvParams &p = pl->cp;
     std::memset(&p, 0, sizeof(p));
+    p.a_tmem_col = a_tmem ? 2 * BN : 0;
     p.off_a = 0;
     p.off_b = p.off_a + a_bytes * stages;
     p.off_stg = p.off_b + b_bytes * stages;
@@ -610,6 +625,9 @@ bool make_plan2(const qconv_desc *d, const Geometry &g, const Plan &pl1, bool ch
     const bool is4 = g.bits == 4;
     const int m_tiles2 = static_cast<int>((g.M + 2 * qc::kBM - 1) / (2 * qc::kBM));
     pl->num_tiles = m_tiles2 * pl1.n_tiles_n;
+    p.a_tmem_col = 0;                                      // (A from TMEM: im2col kernel only)
+    pl->tmem_cols = pow2_cols(2 * BN);
+    p.tmem_cols = pl->tmem_cols;
     const uint32_t a_bytes = static_cast<uint32_t>(qc::kBM * pl1.BK);
     const uint32_t b_bytes = static_cast<uint32_t>(align_up(static_cast<size_t>(BN / 2) * pl1.BK, 1024));
     const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(qc::kBM * pl1.bkp) : 0u;
