@@ -32,6 +32,10 @@ constexpr int kHaloMaxMMA = 18;      // halo kernel: 3x3 taps x 2 plane pairs (C
 // channel-major kernel: 16 epilogue warps (4 per SMSP: the re-quantization is latency- not
 // issue-bound), then the 4 converter warps (4-bit)
 constexpr int kTEpiWarps = 16;
+#ifndef QC_TGROUPS
+#define QC_TGROUPS 2
+#endif
+constexpr int kTGroups = QC_TGROUPS;      // channel-major epilogue: warp groups on alternating tiles
 constexpr int kTProducers = 2;        // TMA issuers: lane 0 of warps 0 and 3 (warp 2: output storer)
 constexpr int kTWarpCvt0 = kWarpEpi0 + kTEpiWarps;
 constexpr int kTThreads8 = 32 * kTWarpCvt0;

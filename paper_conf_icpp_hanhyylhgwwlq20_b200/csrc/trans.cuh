@@ -169,8 +169,8 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(&tfull[i], 1);
-            mbar_init(&tempty[i], kTEpiWarps);
-            mbar_init(&sfull[i], kTEpiWarps);
+            mbar_init(&tempty[i], kTEpiWarps / kTGroups);
+            mbar_init(&sfull[i], kTEpiWarps / kTGroups);
             mbar_init(&sfree[i], 1);
         }
         fence_mbar_init();
@@ -195,8 +195,15 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
                 mbar_wait(&sfull[b], static_cast<uint32_t>(it >> 1) & 1u);
                 tma_store_2d(&ymap, smem + p.off_ystg + b * p.ystg_bytes, c0 * (kInt4 ? 4 : 8) / 8, m0);
                 bulk_commit();
-                bulk_wait_read<1>();                 // the store from buffer b^1 has read its smem
-                if (it > 0) mbar_arrive(&sfree[b ^ 1]);
+                if (kTGroups == 2) {
+                    // buffer b belongs to one epilogue group: release it as soon as its own store
+                    // has read it (the other group keeps working meanwhile)
+                    bulk_wait_read<0>();
+                    mbar_arrive(&sfree[b]);
+                } else {
+                    bulk_wait_read<1>();             // the store from buffer b^1 has read its smem
+                    if (it > 0) mbar_arrive(&sfree[b ^ 1]);
+                }
                 trace_ev(p, 7, it);
             }
             bulk_wait<0>();
@@ -282,14 +289,19 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         const int ew = warp - kWarpEpi0;
         const int quarter = warp & 3;
         const int sub = ew >> 2;                           // 0..3: the 4 warps of a lane quarter
-        // 16-lane group of this warp and its pixel range.  M=128: quarter q holds groups 2q, 2q+1,
-        // two warps per group, 128 pixels each.  M=64 (1-CTA): rows live in lanes 0..15 of each
-        // quarter (group q), the four warps of a quarter take 64 pixels each.
-        const int grp = M64 ? quarter : 2 * quarter + (sub & 1);
+        // kTGroups == 2: warps with sub >> 1 == g take the tiles of parity g (accumulator buffer g,
+        // staging buffer g), so one group's waits overlap the other group's arithmetic instead of
+        // all 16 warps stopping together between tiles.  16-lane group of this warp and its pixel
+        // range: M=128: quarter q holds 16-lane groups 2q, 2q+1; M=64: rows live in lanes 0..15 of
+        // each quarter.
+        constexpr int kWpq = 4 / kTGroups;                 // warps of one quarter per tile
+        const int gsel = kTGroups == 2 ? (sub >> 1) : 0;   // tile parity of this warp
+        const int wq = kTGroups == 2 ? (sub & 1) : sub;    // index among the kWpq warps
+        const int grp = M64 ? quarter : 2 * quarter + (wq & 1);
         const uint32_t lane_base = M64 ? 32u * static_cast<uint32_t>(quarter)
-                                       : 32u * static_cast<uint32_t>(quarter) + 16u * static_cast<uint32_t>(sub & 1);
-        constexpr int kCols = M64 ? kBNp / 4 : kBNp / 2;
-        const int col_begin = M64 ? sub * kCols : (sub >> 1) * kCols;
+                                       : 32u * static_cast<uint32_t>(quarter) + 16u * static_cast<uint32_t>(wq & 1);
+        constexpr int kCols = M64 ? kBNp / kWpq : kBNp / (kWpq / 2);
+        const int col_begin = M64 ? wq * kCols : (wq >> 1) * kCols;
         const int pair = 8 * grp + (lane >> 2);             // channel pair of the tile
         constexpr int kGMask = kRowBytes >= 128 ? 7 : (kRowBytes == 64 ? 3 : 1);
         const uint32_t boff = static_cast<uint32_t>(kInt4 ? pair : 2 * pair);
@@ -297,12 +309,12 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         int cached_c0 = -1;
         TChan ce{}, co{};
         int mode = 2;
-        int it = 0;
+        int it = gsel;
         // channel tile of the CTA's current tile, advanced without divisions
         const int ntn = p.n_tiles_n;
-        const int cstep = static_cast<int>(gridDim.x) % ntn;
-        int cm = static_cast<int>(blockIdx.x) % ntn;
-        for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
+        const int cstep = static_cast<int>((static_cast<int64_t>(gridDim.x) * kTGroups) % ntn);
+        int cm = static_cast<int>((blockIdx.x + static_cast<int64_t>(gsel) * gridDim.x) % ntn);
+        for (int tile = blockIdx.x + gsel * gridDim.x; tile < p.num_tiles; tile += kTGroups * gridDim.x, it += kTGroups) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
             const int c0 = cm * BMc;
@@ -334,7 +346,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             mbar_wait(&sfree[it & 1], (static_cast<uint32_t>(it >> 1) & 1u) ^ 1u);
             const uint32_t ystg = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes;
             const int row0 = col_begin + 2 * (lane & 3);
-            // 64-pixel chunks (latency hidden by the 4 epilogue warps per SMSP)
+            // 64-pixel chunks
 #pragma unroll 1
             for (int t = 0; t < kCols / 64; ++t) {
                 uint32_t va[32];

@@ -36,6 +36,45 @@ __global__ void tmem_read(int iters, long long *out, unsigned *sink) {
     if (warp == 0) { tc_fence_after(); tmem_dealloc(tslot, 512); }
 }
 
+
+__device__ __forceinline__ void tmem_ld_32x32b_x32_p16(uint32_t taddr, uint32_t (&v)[16]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.pack::16b.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, "
+        "%11, %12, %13, %14, %15}, [%16];"
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
+        : "r"(taddr));
+}
+// SHAPE 0: 32x32b.x32 (32 cols), 1: 16x256b.x8 (16 lanes x 64 cols... 32 regs), 2: 32x32b.x16.pack::16b (32 cols -> 16 regs)
+template <int SHAPE>
+__global__ void tmem_read2(int iters, long long *out, unsigned *sink) {
+    __shared__ uint32_t tslot;
+    const int warp = threadIdx.x / 32;
+    if (warp == 0) tmem_alloc(&tslot, 512);
+    tc_fence_before(); __syncthreads(); tc_fence_after();
+    const uint32_t tm = tslot + (static_cast<uint32_t>((warp & 3) * 32 + (SHAPE == 1 ? ((warp >> 2) & 1) * 16 : 0)) << 16);
+    uint32_t acc = 0;
+    __syncthreads();
+    long long t0 = clock64();
+    for (int i = 0; i < iters; ++i) {
+        uint32_t v[32];
+        if (SHAPE == 0) tmem_ld_32x32b_x32(tm + (((i + warp) * 32) & 511), v);
+        else if (SHAPE == 1) tmem_ld_16x256b_x8(tm + (((i + warp) * 64) & 511), v);
+        else { uint32_t u[16]; tmem_ld_32x32b_x32_p16(tm + (((i + warp) * 32) & 511), u);
+#pragma unroll
+               for (int j = 0; j < 16; ++j) v[j] = u[j], v[j + 16] = 0; }
+        tmem_wait_ld();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) acc += v[j];
+    }
+    __syncthreads();
+    long long t1 = clock64();
+    if (threadIdx.x == 0) out[blockIdx.x] = t1 - t0;
+    if (acc == 0x9u) sink[0] = acc;
+    tc_fence_before(); __syncthreads();
+    if (warp == 0) { tc_fence_after(); tmem_dealloc(tslot, 512); }
+}
+
 __global__ void imma(int iters, long long *out, int *sink) {
     int a0 = threadIdx.x * 3 + 1, a1 = a0 ^ 0x55, a2 = a0 * 7, a3 = a0 + 9;
     int b0 = threadIdx.x + 5, b1 = b0 * 3;
@@ -76,6 +115,20 @@ int main() {
             printf("tmem_read warps=%2d batch=%d  cycles=%lld  B/cyc/SM=%.1f\n", warps, batch, h[0],
                    bytes / h[0]);
         }
+    }
+
+    for (int shape : {0, 1, 2}) for (int warps : {4, 8, 16}) {
+        const int iters = 4096;
+        for (int rep = 0; rep < 2; ++rep) {
+            if (shape == 0) tmem_read2<0><<<148, warps * 32>>>(iters, out, sink);
+            else if (shape == 1) tmem_read2<1><<<148, warps * 32>>>(iters, out, sink);
+            else tmem_read2<2><<<148, warps * 32>>>(iters, out, sink);
+        }
+        cudaError_t e = cudaDeviceSynchronize();
+        if (e != cudaSuccess) { printf("err %s\n", cudaGetErrorString(e)); return 1; }
+        cudaMemcpy(h, out, sizeof(h), cudaMemcpyDeviceToHost);
+        const double bytes = static_cast<double>(warps) * iters * 32 * 32 * 4;   // accumulator bytes covered
+        printf("tmem_read2 shape=%d warps=%2d cycles=%lld  acc-B/cyc/SM=%.1f  (32-bit accumulators/cyc/SM=%.1f)\n", shape, warps, h[0], bytes / h[0], bytes / 4 / h[0]);
     }
     for (int warps : {4, 8, 16, 32}) {
         const int iters = 2048;
