@@ -247,36 +247,33 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             RingPos rp;
             const uint32_t sbo = 8u * static_cast<uint32_t>(p.BK);
             const int ksteps = p.BK / 32;
+            // Per tile the accumulator hand-back (tempty) is the critical path: the first K-stage's
+            // operands are waited for and its descriptors formed BEFORE waiting on tempty, so only
+            // the fence and the branch-free issue (ksteps <= 4, predicated) follow it.
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
                 const int buf = it & 1;
                 const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
-                mbar_wait(&tempty[buf], acc_phase ^ 1u);
-                __syncwarp();
-                tc_fence_after();
-                if (lane == 0) trace_ev(p, 2, it);
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * BNp);
                 for (int kb = 0; kb < p.num_kb; ++kb, ++g, rp.next(NS)) {
                     const int stage = rp.stage;
                     mbar_wait(IS4 ? &aready[stage] : &full[stage], rp.phase);
-                    __syncwarp();
-                    tc_fence_after();
-                    if (lane == 0) trace_ev(p, 3, g);
                     const uint32_t w_addr = smem_u32(smem + p.off_b + stage * p.b_stage_bytes);
                     const uint32_t x_addr = smem_u32(smem + p.off_a + stage * p.a_stage_bytes);
                     const uint64_t ad0 = make_smem_desc(w_addr, 16u, sbo, p.sw_layout);
                     const uint64_t bd0 = make_smem_desc(x_addr, 16u, sbo, p.sw_layout);
                     const uint32_t alo = static_cast<uint32_t>(ad0), ahi = static_cast<uint32_t>(ad0 >> 32);
                     const uint32_t blo = static_cast<uint32_t>(bd0), bhi = static_cast<uint32_t>(bd0 >> 32);
-                    if (ksteps == 4) {
-#pragma unroll
-                        for (int k = 0; k < 4; ++k)
-                            mma_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
-                                               (kb | k) != 0 ? 1u : 0u);
-                    } else {
-                        for (int k = 0; k < ksteps; ++k)
-                            mma_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
-                                               (kb | k) != 0 ? 1u : 0u);
+                    if (kb == 0) {
+                        mbar_wait(&tempty[buf], acc_phase ^ 1u);
+                        if (lane == 0) trace_ev(p, 2, it);
                     }
+                    __syncwarp();
+                    tc_fence_after();
+                    if (lane == 0) trace_ev(p, 3, g);
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+                        mma_i8_warp_lo_if(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
+                                          (kb | k) != 0 ? 1u : 0u, k < ksteps ? 1u : 0u);
                     mma_commit_warp(&empty[stage]);
                 }
                 mma_commit_warp(&tfull[buf]);

@@ -75,6 +75,31 @@ __global__ void tmem_read2(int iters, long long *out, unsigned *sink) {
     if (warp == 0) { tc_fence_after(); tmem_dealloc(tslot, 512); }
 }
 
+template <int SHAPE>
+__global__ void tmem_read3(int iters, long long *out, unsigned *sink) {
+    __shared__ uint32_t tslot;
+    const int warp = threadIdx.x / 32;
+    if (warp == 0) tmem_alloc(&tslot, 512);
+    tc_fence_before(); __syncthreads(); tc_fence_after();
+    const uint32_t tm = tslot + (static_cast<uint32_t>((warp & 3) * 32 + (SHAPE == 1 ? ((warp >> 2) & 1) * 16 : 0)) << 16);
+    uint32_t acc = 0;
+    __syncthreads();
+    long long t0 = clock64();
+    for (int i = 0; i < iters; ++i) {
+        uint32_t v[32];
+        if (SHAPE == 0) tmem_ld_32x32b_x32(tm + (((i + warp) * 32) & 511), v);
+        else tmem_ld_16x256b_x8(tm + (((i + warp) * 64) & 511), v);
+        tmem_wait_ld_regs(v);
+        acc ^= v[0] ^ v[31];
+    }
+    __syncthreads();
+    long long t1 = clock64();
+    if (threadIdx.x == 0) out[blockIdx.x] = t1 - t0;
+    if (acc == 0x9u) sink[0] = acc;
+    tc_fence_before(); __syncthreads();
+    if (warp == 0) { tc_fence_after(); tmem_dealloc(tslot, 512); }
+}
+
 __global__ void imma(int iters, long long *out, int *sink) {
     int a0 = threadIdx.x * 3 + 1, a1 = a0 ^ 0x55, a2 = a0 * 7, a3 = a0 + 9;
     int b0 = threadIdx.x + 5, b1 = b0 * 3;
@@ -139,6 +164,18 @@ int main() {
         const double macs = static_cast<double>(warps) * iters * 8 * 16 * 8 * 32;
         printf("imma m16n8k32 warps=%2d cycles=%lld  MAC/cyc/SM=%.0f  (x148 SMs x %.2f GHz = %.0f TOPS)\n",
                warps, h[0], macs / h[0], clk_khz / 1e6, 2 * macs / h[0] * 148 * clk_khz * 1e3 / 1e12);
+    }
+
+    for (int shape : {0, 1}) for (int warps : {4, 8, 16}) {
+        const int iters = 4096;
+        for (int rep = 0; rep < 2; ++rep) {
+            if (shape == 0) tmem_read3<0><<<148, warps * 32>>>(iters, out, sink);
+            else tmem_read3<1><<<148, warps * 32>>>(iters, out, sink);
+        }
+        cudaDeviceSynchronize();
+        cudaMemcpy(h, out, sizeof(h), cudaMemcpyDeviceToHost);
+        const double accs = static_cast<double>(warps) * iters * 32 * 32;
+        printf("tmem_read3 (no ALU) shape=%d warps=%2d cycles=%lld  accumulators/cyc/SM=%.1f\n", shape, warps, h[0], accs / h[0]);
     }
     return 0;
 }

@@ -8,8 +8,8 @@ os.environ["QC_TRACE"] = out
 import torch
 import paper_conf_icpp_hanhyylhgwwlq20_b200 as qc
 import workloads as W
-names = {0: "prod", 2: "mma_tempty", 3: "mma_full", 4: "mma_commit", 5: "epi_tfull", 6: "epi_done",
-         7: "store", 8: "cvt_full", 9: "cvt_arrive"}
+names = {0: "prod", 2: "mma_tempty", 3: "mma_full", 13: "mma_issued", 4: "mma_commit", 5: "epi_tfull",
+         11: "epi_sfree", 6: "epi_done", 14: "epi1_tfull", 15: "epi1_done", 7: "store", 8: "cvt_full", 9: "cvt_arrive"}
 for spec in sys.argv[1:]:
     name, bits = spec.split(':'); bits = int(bits)
     if os.path.exists(out): os.remove(out)
