@@ -153,10 +153,10 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         }
         for (int i = 0; i < 2; ++i) {
             mbar_init(&tfull[i], 1);
-            mbar_init(&tempty[i], kNEpi);
+            mbar_init(&tempty[i], CM ? kNEpi / 2 : kNEpi);
         }
         for (int i = 0; i < kMaxYstg; ++i) {
-            mbar_init(&sfull[i], kNEpi);
+            mbar_init(&sfull[i], CM ? kNEpi / 2 : kNEpi);
             mbar_init(&sfree[i], 1);
         }
         mbar_init(bfull, 1);
@@ -202,9 +202,16 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                                      n0 * kBits / 8 + gi * p.y_gw, 0, p0, img);
                 }
                 bulk_commit();
-                // keep two stores in flight: the previous one has read its buffer -> release it
-                bulk_wait_read<1>();
-                if (it > 0) mbar_arrive(&sfree[bprev]);
+                if (CM && NB == 2) {
+                    // staging buffer b belongs to one epilogue group: release it once its own
+                    // store has read it (the other group keeps working meanwhile)
+                    bulk_wait_read<0>();
+                    mbar_arrive(&sfree[b]);
+                } else {
+                    // keep two stores in flight: the previous one has read its buffer -> release it
+                    bulk_wait_read<1>();
+                    if (it > 0) mbar_arrive(&sfree[bprev]);
+                }
                 bprev = b;
                 if (++b == NB) { b = 0; bphase ^= 1u; }
                 trace_ev(p, 7, it);
@@ -292,10 +299,11 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
             for (int tile = t_first; tile < t_end; tile += t_step, ++it) {
                 const int buf = it & 1;
                 const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
-                mbar_wait(&tempty[buf], acc_phase ^ 1u);
-                if (leader) trace_ev(p, 2, it);
+                // operands first: after the accumulator hand-back only the fence and the issue remain
                 mbar_wait(kCvt ? &hready[stage] : &hfull[stage], phase);
                 if (leader) trace_ev(p, 3, it);
+                mbar_wait(&tempty[buf], acc_phase ^ 1u);
+                if (leader) trace_ev(p, 2, it);
                 __syncwarp();
                 tc_fence_after();
                 if (leader) trace_ev(p, 1, it);
@@ -347,7 +355,9 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         constexpr int kRowBytes = 64 * (kInt4 ? 4 : 8) / 8;
         constexpr int kGMask = kRowBytes >= 128 ? 7 : (kRowBytes == 64 ? 3 : 1);
         const uint32_t lane_base = 32u * static_cast<uint32_t>(quarter);
-        const int col_begin = sub * 64;
+        // two warp groups (sub >> 1) take alternating tiles; a warp covers 128 pixel columns
+        const int gsel = sub >> 1;
+        const int col_begin = (sub & 1) * 128;
         const int pair = 8 * quarter + (lane >> 2);
         const uint32_t boff = static_cast<uint32_t>(kInt4 ? pair : 2 * pair);
         const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
@@ -372,26 +382,28 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
         }
         const uint32_t taddr0 = tmem_base + (lane_base << 16) + static_cast<uint32_t>(col_begin);
         const int row0 = col_begin + 2 * (lane & 3);
-        int it = 0;
-        int sb = 0;
-        uint32_t sphase = 0;
-        for (int tile = t_first; tile < t_end; tile += t_step, ++it) {
+        int it = gsel;
+        for (int tile = t_first + gsel * t_step; tile < t_end; tile += 2 * t_step, it += 2) {
             const int buf = it & 1;
             const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
+            const int sb = it % NB;
+            const uint32_t sphase = static_cast<uint32_t>(it / NB) & 1u;
             mbar_wait(&tfull[buf], acc_phase);
             tc_fence_after();
             if (ew == 0 && lane == 0) trace_ev(p, 5, it);
             mbar_wait(&sfree[sb], sphase ^ 1u);
             if (ew == 0 && lane == 0) trace_ev(p, 10, it);
             const uint32_t ystg = ystg_base + static_cast<uint32_t>(sb) * p.ystg_bytes;
-            uint32_t va[32];
-            tmem_ld_16x256b_x8(taddr0 + static_cast<uint32_t>(buf * 256), va);
-            // the multipliers re-enter the loop as plain 32-bit registers: hoisted out of it as
-            // sign-extended 64-bit values they turned every product into a 64x64 multiply
-            asm volatile("" : "+r"(ce.m), "+r"(co.m));
-            tmem_wait_ld_regs(va);
-            if (ew == 0 && lane == 0) trace_ev(p, 13, it);
-            t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, va, ystg, row0, boff);
+#pragma unroll 1
+            for (int t = 0; t < 2; ++t) {
+                uint32_t va[32];
+                tmem_ld_16x256b_x8(taddr0 + static_cast<uint32_t>(buf * 256 + 64 * t), va);
+                // the multipliers re-enter the loop as plain 32-bit registers: hoisted out of it as
+                // sign-extended 64-bit values they turned every product into a 64x64 multiply
+                asm volatile("" : "+r"(ce.m), "+r"(co.m));
+                tmem_wait_ld_regs(va);
+                t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, va, ystg, row0 + 64 * t, boff);
+            }
             if (ew == 0 && lane == 0) trace_ev(p, 14, it);
             tc_fence_before();
             fence_proxy_async_smem();                 // staging writes -> visible to the TMA store
@@ -400,7 +412,6 @@ qconv_halo_kernel(const __grid_constant__ CUtensorMap hmap, const __grid_constan
                 mbar_arrive(&tempty[buf]);
                 mbar_arrive(&sfull[sb]);
             }
-            if (++sb == NB) { sb = 0; sphase ^= 1u; }
             if (ew == 0 && lane == 0) trace_ev(p, 6, it);
         }
     } else if (!CM && warp >= kEpi0 && warp < kEpi0 + kNumEpiWarps) {
