@@ -81,6 +81,23 @@ __device__ __forceinline__ void mma2_i8_warp_lo(uint32_t d_tmem, uint32_t alo, u
         "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "r"(accumulate)
         : "memory");
 }
+// Same, issued only when `active` is non-zero: a fully unrolled, branch-free run (see
+// ptx.cuh mma_i8_warp_lo_if: branch-guarded MMAs each wait for their own operand moves).
+__device__ __forceinline__ void mma2_i8_warp_lo_if(uint32_t d_tmem, uint32_t alo, uint32_t ahi, uint32_t blo,
+                                                   uint32_t bhi, uint32_t idesc, uint32_t accumulate,
+                                                   uint32_t active) {
+    asm volatile(
+        "{\n\t.reg .pred p, e, q;\n\t.reg .b64 da, db;\n\t"
+        "setp.ne.b32 p, %6, 0;\n\t"
+        "setp.ne.b32 q, %7, 0;\n\t"
+        "mov.b64 da, {%1, %2};\n\t"
+        "mov.b64 db, {%3, %4};\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "and.pred e, e, q;\n\t"
+        "@e tcgen05.mma.cta_group::2.kind::i8 [%0], da, db, %5, p;\n\t}" ::"r"(d_tmem),
+        "r"(alo), "r"(ahi), "r"(blo), "r"(bhi), "r"(idesc), "r"(accumulate), "r"(active)
+        : "memory");
+}
 // commit to the barrier at the same offset in both CTAs of the pair
 __device__ __forceinline__ void mma2_commit_mc_warp(uint64_t *bar) {
     asm volatile(
@@ -251,9 +268,10 @@ qconv_fwd2_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constan
                                                         p.sw_layout);
                     const uint32_t alo = static_cast<uint32_t>(ad0), ahi = static_cast<uint32_t>(ad0 >> 32);
                     const uint32_t blo = static_cast<uint32_t>(bd0), bhi = static_cast<uint32_t>(bd0 >> 32);
-                    for (int k = 0; k < ksteps; ++k)
-                        mma2_i8_warp_lo(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
-                                        (kb | k) != 0 ? 1u : 0u);
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+                        mma2_i8_warp_lo_if(d_tmem, alo + 2u * k, ahi, blo + 2u * k, bhi, p.idesc,
+                                           (kb | k) != 0 ? 1u : 0u, k < ksteps ? 1u : 0u);
                     mma2_commit_mc_warp(&empty[stage]);
                     if (lane == 0) trace_ev2(p, 3, gs, 0);
                     ++gs;
