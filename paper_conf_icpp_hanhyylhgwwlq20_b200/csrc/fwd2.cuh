@@ -15,6 +15,9 @@
 //   tfull[b] (both)   : accumulator b complete -- multicast commit
 //   tempty[b](leader) : both CTAs' epilogue warps drained accumulator b -- local + remote arrives
 #pragma once
+#ifndef QC_REMOTE_RELEASE_CLUSTER
+#define QC_REMOTE_RELEASE_CLUSTER 0
+#endif
 #include "epilogue.cuh"
 
 namespace qc {
@@ -54,11 +57,19 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t *bar, uint32_t parity
     }
 }
 // Remote arrive with the default (.release.cta) semantics, as CUTLASS's ClusterBarrier does: a
-// .release.cluster arrive costs the converter warps ~0.5 us per stage (measured, trace_fwd2.py).
+// .release.cluster arrive costs the converter warps ~0.5 us per stage (measured, trace_fwd2.py;
+// re-measured late in round 2 with -DQC_REMOTE_RELEASE_CLUSTER=1: 4-bit pair family 537 -> 913 us
+// per A4W4 step, 8-bit 433 -> 455).
 // The data the leader's MMA then reads stays in this CTA's shared memory, made visible to the
 // async proxy by the preceding fence.proxy.async.
 __device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+#if QC_REMOTE_RELEASE_CLUSTER
+    // release at cluster scope: the peer's shared-memory / TMEM work before the arrive is
+    // ordered before the leader's acquire.cluster wait (PTX memory model, cross-CTA)
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+#else
     asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+#endif
 }
 __device__ __forceinline__ void tmem_alloc2(uint32_t *dst_smem, uint32_t ncols) {
     asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
