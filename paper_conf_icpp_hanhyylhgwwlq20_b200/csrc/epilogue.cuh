@@ -35,7 +35,9 @@ constexpr int kTEpiWarps = 16;
 #ifndef QC_TGROUPS
 #define QC_TGROUPS 2
 #endif
-constexpr int kTGroups = QC_TGROUPS;      // channel-major epilogue: warp groups on alternating tiles
+// channel-major epilogue: warp groups on round-robin tiles, one accumulator (kTBNp pixels) each
+constexpr int kTGroups = QC_TGROUPS;
+constexpr int kTBNp = kTGroups == 4 ? 128 : 256;
 constexpr int kTProducers = 2;        // TMA issuers: lane 0 of warps 0 and 3 (warp 2: output storer)
 constexpr int kTWarpCvt0 = kWarpEpi0 + kTEpiWarps;
 constexpr int kTThreads8 = 32 * kTWarpCvt0;

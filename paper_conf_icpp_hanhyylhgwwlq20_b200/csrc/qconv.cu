@@ -877,7 +877,7 @@ bool make_trans_plan(const qconv_desc *d, const Geometry &g, int bmc_req, bool c
         if (d->k % bmc_req) return false;
         BMc = bmc_req;
     }
-    const int BNp = 256;
+    const int BNp = qc::kTBNp;                               // pixels per tile (trans.cuh)
     const int BK = choose_bk(d->c);
     const int bkp = is4 ? BK / 2 : BK;
     const int n_tiles_n = d->k / BMc;
@@ -890,7 +890,7 @@ bool make_trans_plan(const qconv_desc *d, const Geometry &g, int bmc_req, bool c
     const uint32_t b_bytes = static_cast<uint32_t>(BMc * BK);      // weights
     const uint32_t stg_bytes = is4 ? static_cast<uint32_t>(BNp * bkp) : 0u;
     const uint32_t per_stage = a_bytes + b_bytes + stg_bytes;
-    const uint32_t fixed = 2u * ystg_one + 2048u;
+    const uint32_t fixed = static_cast<uint32_t>(qc::kTGroups) * ystg_one + 2048u;
     if (fixed + 2 * per_stage > 227u * 1024u) return false;
     int stages = std::min(static_cast<int>((227u * 1024u - fixed) / per_stage), 16);
     qc::ConvParams &p = pl->cp;
@@ -922,14 +922,14 @@ bool make_trans_plan(const qconv_desc *d, const Geometry &g, int bmc_req, bool c
     p.y_gw = row_bytes;
     p.y_gmask = row_bytes >= 128 ? 7 : (row_bytes == 64 ? 3 : 1);   // staging swizzled like the TMA store
     p.n_ygroups = 1;
-    p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + 2u * ystg_one, 16));
+    p.off_par = static_cast<uint32_t>(align_up(p.off_ystg + static_cast<uint32_t>(qc::kTGroups) * ystg_one, 16));
     p.off_bar = static_cast<uint32_t>(align_up(p.off_par, 8));
-    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 8) * 8 + 16);
+    const uint32_t bar_bytes = static_cast<uint32_t>((3 * stages + 16) * 8 + 16);
     pl->smem_bytes = p.off_bar + bar_bytes + 1024u;
     if (pl->smem_bytes > 227u * 1024u) return false;
     p.idesc = qc::make_idesc_i8(static_cast<uint32_t>(BMc), static_cast<uint32_t>(BNp),
                                 dtype_signed(d->w_t), act_signed(d));
-    pl->tmem_cols = pow2_cols(2 * BNp);
+    pl->tmem_cols = pow2_cols(qc::kTGroups * BNp);
     p.tmem_cols = pl->tmem_cols;
     p.y_zero = d->y_zero; p.clamp_lo = d->clamp_lo; p.clamp_hi = d->clamp_hi;
     p.need_clamp = (d->clamp_lo > dtype_min(d->y_t) || d->clamp_hi < dtype_max(d->y_t)) ? 1 : 0;

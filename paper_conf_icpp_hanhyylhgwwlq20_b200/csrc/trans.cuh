@@ -142,8 +142,10 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
     const int lane = threadIdx.x & 31;
     const int NS = p.stages;
     constexpr int BMc = M64 ? 64 : 128;   // output channels per tile (UMMA M)
-    constexpr int kBNp = 256;             // output pixels per tile (UMMA N)
+    constexpr int kBNp = kTBNp;           // output pixels per tile (UMMA N)
     constexpr int BNp = kBNp;
+    constexpr int kNB = kTGroups;         // accumulator buffers = staging buffers = epilogue groups
+    constexpr int kLgNB = kNB == 4 ? 2 : 1;
     constexpr bool kInt4 = (OUT == OUT_U4 || OUT == OUT_S4);
     constexpr int kRowBytes = BMc * (kInt4 ? 4 : 8) / 8;      // staging row = one pixel
 
@@ -151,11 +153,11 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
     uint64_t *full = bars;
     uint64_t *empty = bars + NS;
     uint64_t *aready = bars + 2 * NS;
-    uint64_t *tfull = bars + 3 * NS;
-    uint64_t *tempty = bars + 3 * NS + 2;
-    uint64_t *sfull = bars + 3 * NS + 4;    // [2] epilogue warps -> storer: staging buffer written
-    uint64_t *sfree = bars + 3 * NS + 6;    // [2] storer -> epilogue warps: its TMA store has read it
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 8);
+    uint64_t *tfull = bars + 3 * NS;        // [kNB] MMA -> epilogue group: accumulator written
+    uint64_t *tempty = bars + 3 * NS + 4;   // [kNB] epilogue group -> MMA: accumulator read
+    uint64_t *sfull = bars + 3 * NS + 8;    // [kNB] epilogue group -> storer: staging buffer written
+    uint64_t *sfree = bars + 3 * NS + 12;   // [kNB] storer -> epilogue group: its TMA store has read it
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 3 * NS + 16);
 
     griddep_launch_dependents();
     if (warp == kWarpTMA && lane == 0) {
@@ -167,7 +169,7 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             mbar_init(&empty[i], 1);
             mbar_init(&aready[i], kNumCvtWarps);
         }
-        for (int i = 0; i < 2; ++i) {
+        for (int i = 0; i < kNB; ++i) {
             mbar_init(&tfull[i], 1);
             mbar_init(&tempty[i], kTEpiWarps / kTGroups);
             mbar_init(&sfull[i], kTEpiWarps / kTGroups);
@@ -189,21 +191,16 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         if (warp == 2 && lane == 0) {
             int it = 0;
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
-                const int b = it & 1;
+                const int b = it & (kNB - 1);
                 const int m0 = (tile / p.n_tiles_n) * BNp;
                 const int c0 = (tile % p.n_tiles_n) * BMc;
-                mbar_wait(&sfull[b], static_cast<uint32_t>(it >> 1) & 1u);
+                mbar_wait(&sfull[b], static_cast<uint32_t>(it >> kLgNB) & 1u);
                 tma_store_2d(&ymap, smem + p.off_ystg + b * p.ystg_bytes, c0 * (kInt4 ? 4 : 8) / 8, m0);
                 bulk_commit();
-                if (kTGroups == 2) {
-                    // buffer b belongs to one epilogue group: release it as soon as its own store
-                    // has read it (the other group keeps working meanwhile)
-                    bulk_wait_read<0>();
-                    mbar_arrive(&sfree[b]);
-                } else {
-                    bulk_wait_read<1>();             // the store from buffer b^1 has read its smem
-                    if (it > 0) mbar_arrive(&sfree[b ^ 1]);
-                }
+                // buffer b belongs to one epilogue group: release it as soon as its own store
+                // has read it (the other groups keep working meanwhile)
+                bulk_wait_read<0>();
+                mbar_arrive(&sfree[b]);
                 trace_ev(p, 7, it);
             }
             bulk_wait<0>();
@@ -251,8 +248,8 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
             // operands are waited for and its descriptors formed BEFORE waiting on tempty, so only
             // the fence and the branch-free issue (ksteps <= 4, predicated) follow it.
             for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x, ++it) {
-                const int buf = it & 1;
-                const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
+                const int buf = it & (kNB - 1);
+                const uint32_t acc_phase = static_cast<uint32_t>(it >> kLgNB) & 1u;
                 const uint32_t d_tmem = tmem_base + static_cast<uint32_t>(buf * BNp);
                 for (int kb = 0; kb < p.num_kb; ++kb, ++g, rp.next(NS)) {
                     const int stage = rp.stage;
@@ -286,77 +283,90 @@ qconv_t_kernel(const __grid_constant__ CUtensorMap xmap, const __grid_constant__
         const int ew = warp - kWarpEpi0;
         const int quarter = warp & 3;
         const int sub = ew >> 2;                           // 0..3: the 4 warps of a lane quarter
-        // kTGroups == 2: warps with sub >> 1 == g take the tiles of parity g (accumulator buffer g,
-        // staging buffer g), so one group's waits overlap the other group's arithmetic instead of
-        // all 16 warps stopping together between tiles.  16-lane group of this warp and its pixel
-        // range: M=128: quarter q holds 16-lane groups 2q, 2q+1; M=64: rows live in lanes 0..15 of
-        // each quarter.
-        constexpr int kWpq = 4 / kTGroups;                 // warps of one quarter per tile
-        const int gsel = kTGroups == 2 ? (sub >> 1) : 0;   // tile parity of this warp
-        const int wq = kTGroups == 2 ? (sub & 1) : sub;    // index among the kWpq warps
-        const int grp = M64 ? quarter : 2 * quarter + (wq & 1);
-        const uint32_t lane_base = M64 ? 32u * static_cast<uint32_t>(quarter)
-                                       : 32u * static_cast<uint32_t>(quarter) + 16u * static_cast<uint32_t>(wq & 1);
-        constexpr int kCols = M64 ? kBNp / kWpq : kBNp / (kWpq / 2);
-        const int col_begin = M64 ? wq * kCols : (wq >> 1) * kCols;
-        const int pair = 8 * grp + (lane >> 2);             // channel pair of the tile
+        // kTGroups epilogue groups take the tiles round robin (group g: tiles it = g mod kTGroups,
+        // accumulator and staging buffer g), so one group's waits overlap the other groups'
+        // arithmetic instead of all 16 warps stopping together between tiles.  M=128: quarter q
+        // holds 16-lane groups 2q, 2q+1; M=64: rows live in lanes 0..15 of each quarter.
+        //  2 groups: a warp covers one 16-lane group, 256 pixels (M=64: 128 pixels)
+        //  4 groups: a warp covers its whole quarter (both 16-lane groups at M=128), 128 pixels
+        const int gsel = kTGroups == 4 ? sub : (sub >> 1);
+        const int wq = kTGroups == 4 ? 0 : (sub & 1);
+        constexpr int kNH = (!M64 && kTGroups == 4) ? 2 : 1;     // 16-lane groups per warp
+        constexpr int kCols = (M64 && kTGroups == 2) ? kBNp / 2 : kBNp;
+        const int col_begin = (M64 && kTGroups == 2) ? wq * kCols : 0;
         constexpr int kGMask = kRowBytes >= 128 ? 7 : (kRowBytes == 64 ? 3 : 1);
-        const uint32_t boff = static_cast<uint32_t>(kInt4 ? pair : 2 * pair);
+        int pair[kNH];
+        uint32_t lane_base[kNH];
+#pragma unroll
+        for (int hh = 0; hh < kNH; ++hh) {
+            const int grp = M64 ? quarter : 2 * quarter + (kTGroups == 4 ? hh : (wq & 1));
+            pair[hh] = 8 * grp + (lane >> 2);               // channel pair of the tile
+            lane_base[hh] = M64 ? 32u * static_cast<uint32_t>(quarter) : 16u * static_cast<uint32_t>(grp);
+        }
         const uint32_t ystg_base = smem_u32(smem + p.off_ystg);
         int cached_c0 = -1;
-        TChan ce{}, co{};
-        int mode = 2;
+        TChan ce[kNH], co[kNH];
+        int mode[kNH];
+#pragma unroll
+        for (int hh = 0; hh < kNH; ++hh) { ce[hh] = TChan{}; co[hh] = TChan{}; mode[hh] = 2; }
         int it = gsel;
         // channel tile of the CTA's current tile, advanced without divisions
         const int ntn = p.n_tiles_n;
         const int cstep = static_cast<int>((static_cast<int64_t>(gridDim.x) * kTGroups) % ntn);
         int cm = static_cast<int>((blockIdx.x + static_cast<int64_t>(gsel) * gridDim.x) % ntn);
         for (int tile = blockIdx.x + gsel * gridDim.x; tile < p.num_tiles; tile += kTGroups * gridDim.x, it += kTGroups) {
-            const int buf = it & 1;
-            const uint32_t acc_phase = static_cast<uint32_t>(it >> 1) & 1u;
+            const int buf = it & (kNB - 1);
+            const uint32_t acc_phase = static_cast<uint32_t>(it >> kLgNB) & 1u;
             const int c0 = cm * BMc;
             cm += cstep;
             if (cm >= ntn) cm -= ntn;
             if (c0 != cached_c0) {
-                const int ke = c0 + 2 * pair, ko = ke + 1;
-                int nee, neo;
-                bool be, bo;
-                t_chan_params(p, ke, ke < p.K, ce, nee, be);
-                t_chan_params(p, ko, ko < p.K, co, neo, bo);
-                const unsigned act = 0xffffffffu;
-                const bool all_fast = __ballot_sync(act, be && bo && nee >= 33 && nee <= 52 && neo >= 33 && neo <= 52) == act;
-                const bool all_mid = __ballot_sync(act, be && bo && nee >= 20 && nee <= 50 && neo >= 20 && neo <= 50 &&
-                                                            mid_multiplier_ok(ce.m) && mid_multiplier_ok(co.m)) == act;
-                mode = all_fast ? 0 : (all_mid ? 1 : 2);
-                if (mode == 1) {
-                    const int T = max(33, __reduce_max_sync(act, max(nee, neo)));
-                    t_chan_mid(p, ce, nee, T);
-                    t_chan_mid(p, co, neo, T);
+#pragma unroll
+                for (int hh = 0; hh < kNH; ++hh) {
+                    const int ke = c0 + 2 * pair[hh], ko = ke + 1;
+                    int nee, neo;
+                    bool be, bo;
+                    t_chan_params(p, ke, ke < p.K, ce[hh], nee, be);
+                    t_chan_params(p, ko, ko < p.K, co[hh], neo, bo);
+                    const unsigned act = 0xffffffffu;
+                    const bool all_fast = __ballot_sync(act, be && bo && nee >= 33 && nee <= 52 && neo >= 33 && neo <= 52) == act;
+                    const bool all_mid = __ballot_sync(act, be && bo && nee >= 20 && nee <= 50 && neo >= 20 && neo <= 50 &&
+                                                                mid_multiplier_ok(ce[hh].m) && mid_multiplier_ok(co[hh].m)) == act;
+                    mode[hh] = all_fast ? 0 : (all_mid ? 1 : 2);
+                    if (mode[hh] == 1) {
+                        const int T = max(33, __reduce_max_sync(act, max(nee, neo)));
+                        t_chan_mid(p, ce[hh], nee, T);
+                        t_chan_mid(p, co[hh], neo, T);
+                    }
                 }
                 cached_c0 = c0;
             }
             mbar_wait(&tfull[buf], acc_phase);
             tc_fence_after();
             if (ew == 0 && lane == 0) trace_ev(p, 5, it);
-            const uint32_t taddr = tmem_base + (lane_base << 16) + static_cast<uint32_t>(buf * kBNp + col_begin);
-            // staging buffer it&1 is free once the store of tile it-2 has read it
-            mbar_wait(&sfree[it & 1], (static_cast<uint32_t>(it >> 1) & 1u) ^ 1u);
-            const uint32_t ystg = ystg_base + static_cast<uint32_t>(it & 1) * p.ystg_bytes;
+            // staging buffer `buf` is free once the store of tile it - kNB has read it
+            mbar_wait(&sfree[buf], acc_phase ^ 1u);
+            const uint32_t ystg = ystg_base + static_cast<uint32_t>(buf) * p.ystg_bytes;
             const int row0 = col_begin + 2 * (lane & 3);
-            // 64-pixel chunks
+#pragma unroll
+            for (int hh = 0; hh < kNH; ++hh) {
+                const uint32_t taddr = tmem_base + (lane_base[hh] << 16) + static_cast<uint32_t>(buf * kBNp + col_begin);
+                const uint32_t boff = static_cast<uint32_t>(kInt4 ? pair[hh] : 2 * pair[hh]);
+                // 64-pixel chunks
 #pragma unroll 1
-            for (int t = 0; t < kCols / 64; ++t) {
-                uint32_t va[32];
-                tmem_ld_16x256b_x8(taddr + static_cast<uint32_t>(t * 64), va);
-                tmem_wait_ld_regs(va);
-                t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode, ce, co, va, ystg, row0 + 64 * t, boff);
+                for (int t = 0; t < kCols / 64; ++t) {
+                    uint32_t va[32];
+                    tmem_ld_16x256b_x8(taddr + static_cast<uint32_t>(t * 64), va);
+                    tmem_wait_ld_regs(va);
+                    t_pairs_mode<OUT, kRowBytes, kGMask>(p, mode[hh], ce[hh], co[hh], va, ystg, row0 + 64 * t, boff);
+                }
             }
             tc_fence_before();
             fence_proxy_async_smem();                 // staging writes -> visible to the TMA store
             __syncwarp();
             if (lane == 0) {
                 mbar_arrive(&tempty[buf]);
-                mbar_arrive(&sfull[it & 1]);
+                mbar_arrive(&sfull[buf]);
             }
             if (ew == 0 && lane == 0) trace_ev(p, 6, it);
         }
