@@ -121,7 +121,7 @@ def stem_scale(bits: int) -> float:
 class Trunk:
     """The 53 ResNet-50 conv layers resident on one GPU (C5's per-rank shard)."""
 
-    def __init__(self, bits: int, batch: int, device, dist_ctx=None, rank: int = 0):
+    def __init__(self, bits: int, batch: int, device, dist_ctx=None, rank: int = 0, stem_dtype: str = "bf16"):
         import torch
         import paper_conf_icpp_hanhyylhgwwlq20_b200 as qc
         self.qc = qc
@@ -158,6 +158,11 @@ class Trunk:
         stem = specs[0][0]
         self.x_float = torch.relu(torch.randn((batch, stem.h, stem.w, stem.c), generator=g,
                                               device=device, dtype=torch.float32))
+        # the image as the stem reads it: bf16 (default; half the bytes over PCIe and HBM, the
+        # quantize takes the exact fp32 value of each bf16) or fp32
+        self.stem_dtype = stem_dtype
+        if stem_dtype == "bf16":
+            self.x_float = self.x_float.to(torch.bfloat16)
         self.s_in = stem_scale(bits)
         # the stem (7x7/s2, C=3) takes the fp32 image: qconv2d_forward_quantize runs it as one
         # kernel (the fp32 rows are quantized inside it, straight into its space-to-depth
@@ -200,8 +205,8 @@ class Trunk:
                 src = cur
             assert src.shape[1] == d.h and src.shape[2] == d.w, cs.name
             ops, nbytes = layer_algorithmic(cs, bits)
-            if i == 0:                      # the stem reads the fp32 image, not codes
-                nbytes += cs.n * cs.h * cs.w * cs.c * (4 - bits / 8)
+            if i == 0:                      # the stem reads the float image, not codes
+                nbytes += cs.n * cs.h * cs.w * cs.c * (self.x_float.element_size() - bits / 8)
             plan = qc.qconv_debug_plan_quantize(d) if i == 0 else qc.qconv_debug_plan(d)
             self.layers.append(dict(name=cs.name, shape=cs, desc=d, w=w_prep, bias=pb[0], m=pb[1],
                                     n=pb[2], x=src, y=y, ops=ops, bytes=nbytes, plan=plan))
@@ -320,10 +325,11 @@ class OracleTrunk:
                                   clamp_lo=lp.clamp_lo, clamp_hi=lp.clamp_hi, bias=lp.bias,
                                   mult=m, shift=n)
 
-    def chain(self, xf, res2, layer_subset=None):
-        """xf: fp32 [1,224,224,3] stem input, res2: packed res2 input codes [1,56,56,*].
-        Returns (outputs per layer -- None where skipped --, ops done)."""
-        xq = self.oracle.quantize(xf, stem_scale(self.bits), 0, self.x_t, c_pad=self.specs[0][1])
+    def chain(self, xf, res2, layer_subset=None, bf16=False):
+        """xf: fp32 [1,224,224,3] stem input (bf16=True: its uint16 bf16 bit patterns), res2:
+        packed res2 input codes [1,56,56,*].  Returns (outputs per layer -- None where
+        skipped --, ops done)."""
+        xq = self.oracle.quantize(xf, stem_scale(self.bits), 0, self.x_t, c_pad=self.specs[0][1], bf16=bf16)
         subset = range(len(self.specs)) if layer_subset is None else layer_subset
         cur = block_in = None
         outs, ops = [], 0
@@ -373,13 +379,16 @@ class OracleTrunk:
 def verify_trunk(trunk: Trunk, images, ot: OracleTrunk = None):
     """Bench self-check (after the timed region): the rank's images `images` through the
     oracle chain; every layer's GPU output bytes of those images must equal the oracle's."""
+    import torch
     if ot is None:
         ot = OracleTrunk(trunk.bits)
     t0 = time.perf_counter()
     bad = []
     for img in images:
-        xf = trunk.x_float[img:img + 1].cpu().numpy()
-        outs, _ = ot.chain(xf, trunk.res2_host[img:img + 1])
+        xt = trunk.x_float[img:img + 1].cpu()
+        bf16 = xt.dtype == torch.bfloat16
+        xf = xt.view(torch.int16).numpy().view(np.uint16) if bf16 else xt.numpy()
+        outs, _ = ot.chain(xf, trunk.res2_host[img:img + 1], bf16=bf16)
         for L, ref in zip(trunk.layers, outs):
             got = L["y"][img:img + 1].cpu().numpy()
             if not np.array_equal(got, ref):
@@ -466,7 +475,7 @@ def run_trunk(args):
         auto = os.path.join(ROOT, "plans", f"resnet50_trunk_a{args.bits}_b{per_gpu}.json")
         plans_path = auto if os.path.exists(auto) else None
     n_plans = tuning.load_plans(plans_path) if plans_path else 0
-    trunk = Trunk(args.bits, per_gpu, device, dist_ctx, rank=rank)
+    trunk = Trunk(args.bits, per_gpu, device, dist_ctx, rank=rank, stem_dtype=args.stem_dtype)
     plans_note = (f"profile-run table {os.path.relpath(plans_path, ROOT)} ({n_plans} shapes)"
                   if n_plans else "default rule")
     if args.tune:
@@ -617,7 +626,9 @@ def run_trunk(args):
             "config": {"workload": f"resnet50_conv_trunk_a{args.bits}w{args.bits}",
                        "global_batch": global_batch, "per_gpu_batch": per_gpu,
                        "layers": len(trunk.layers), "parallelism": f"dp{world} (batch shards)",
-                       "l2": "inputs > L2: 154 MB fp32 stem input and ~2.4 GB of trunk traffic per step "
+                       "stem_input": f"{trunk.stem_dtype} NHWC image, quantized inside the stem kernel",
+                       "l2": f"inputs > L2: {trunk.x_float.numel() * trunk.x_float.element_size() / 1e6:.0f} MB "
+                             f"{trunk.stem_dtype} stem input and ~2.4 GB of trunk traffic per step "
                              "(at 256 images per GPU)",
                        "graph": "one CUDA graph per step (PDL between the conv kernels), replayed",
                        "plans": plans_note},
@@ -877,6 +888,8 @@ def main():
     ap.add_argument("--plans", default="", help="tile-search table to apply ('' = plans/<workload>.json "
                                                 "if present, 'none' = the default rule)")
     ap.add_argument("--save-plans", default="", help="write the --tune results to this table")
+    ap.add_argument("--stem-dtype", default="bf16", choices=("bf16", "fp32"),
+                    help="dtype of the image the stem quantizes (and of the e2e H2D copy)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-verify", action="store_true")

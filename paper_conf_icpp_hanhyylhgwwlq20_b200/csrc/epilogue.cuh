@@ -90,6 +90,7 @@ struct ConvParams {
     float q_inv_s, q_flo, q_fhi;
     int32_t q_z, q_qmin, q_qmax;
     int32_t f_w, f_c, f_pad_h, f_pad_w, f_rowbytes;
+    int32_t bf16;                     // fused stem: the input image is bf16 (else fp32)
     int32_t a_tmem_col;           // > 0 (im2col, 4-bit): the widened A operand goes to TMEM here
     int32_t b_res;                    // channel-major: the CTA's weights resident at off_bres
     const uint8_t *x_lin;             // channel-major 4-bit, 1x1/s1/p0, one K chunk: activations read

@@ -62,7 +62,13 @@ __device__ __forceinline__ void f32_s2d_pixel(const ConvParams &p, const uint32_
 #pragma unroll
         for (int cc = 0; cc < C; ++cc) {
             float v;
-            asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr[blk] + 4u * cc));
+            if (p.bf16) {     // bf16 input: the exact fp32 value is the bf16 bits << 16
+                uint32_t u;
+                asm volatile("ld.shared.u16 %0, [%1];" : "=r"(u) : "r"(addr[blk] + 2u * cc));
+                v = __uint_as_float(u << 16);
+            } else {
+                asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr[blk] + 4u * cc));
+            }
             code[blk * C + cc] = f32_q(p, v);
         }
     }
@@ -88,7 +94,8 @@ __device__ __forceinline__ uint32_t f32_s2d_offsets(const ConvParams &p, int j, 
     for (int blk = 0; blk < 4; ++blk) {
         const int ww = 2 * j + (blk & 1) - p.f_pad_w;
         const bool in = ww >= 0 && ww < p.f_w;
-        off[blk] = (blk >> 1) * static_cast<uint32_t>(p.f_rowbytes) + 4u * static_cast<uint32_t>((in ? ww : 0) * p.f_c);
+        off[blk] = (blk >> 1) * static_cast<uint32_t>(p.f_rowbytes) +
+                   (p.bf16 ? 2u : 4u) * static_cast<uint32_t>((in ? ww : 0) * p.f_c);
         ok |= in ? (1u << blk) : 0u;
     }
     return ok;

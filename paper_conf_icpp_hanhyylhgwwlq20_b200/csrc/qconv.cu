@@ -1265,6 +1265,7 @@ qc_status forward_impl(const qconv_desc *d, bool dequant, const void *x, const v
 // (halo.cuh F32); any other layer quantizes into the workspace, then runs qconv2d_forward.
 struct QExec {
     bool fused;
+    int esz;                  // input element bytes: 4 (fp32) or 2 (bf16)
     Exec ex;                  // fused: the s2d exec descriptor; else the codes' exec descriptor
     Plan pl;                  // fused: the halo plan with fp32 staging
     qconv_desc dq;            // fallback: the descriptor of the quantized codes
@@ -1275,6 +1276,7 @@ struct QExec {
 qc_status derive_qexec(const qconv_desc *d, qc_ftype xt, QExec *qx) {
     if (!d) return QC_ERR_INVALID_ARG;
     if (xt != QC_F32 && xt != QC_BF16) return QC_ERR_INVALID_ARG;
+    qx->esz = xt == QC_BF16 ? 2 : 4;
     qconv_desc dv = *d;                      // codes of any 4-bit c live in bytes in the s2d form
     dv.x_t = byte_container(d->x_t);
     Geometry gv;
@@ -1282,7 +1284,7 @@ qc_status derive_qexec(const qconv_desc *d, qc_ftype xt, QExec *qx) {
     if (s != QC_OK) return s;
     if (!is_int_input(d->x_t)) return QC_ERR_INVALID_ARG;
     const bool s2d_ok = d->stride_h == 2 && d->stride_w == 2 && d->dil_h == 1 && d->dil_w == 1 &&
-                        4 * d->c <= 16 && d->w_zero == nullptr && d->x_zero == 0 && xt == QC_F32 &&
+                        4 * d->c <= 16 && d->w_zero == nullptr && d->x_zero == 0 &&
                         (static_cast<int64_t>(d->w) * d->c) % 4 == 0 && static_cast<int64_t>(d->w) * d->c <= 1024 &&
                         is_packed_out(d->y_t);
     qx->fused = false;
@@ -1302,7 +1304,7 @@ qc_status derive_qexec(const qconv_desc *d, qc_ftype xt, QExec *qx) {
             ex.ws_total = ex.wprep_needed ? align_up(ex.prep_bytes, 256) : 0;
             // the fused stem runs the channel-major halo when it is eligible (K = 64), unless a
             // plan choice for `d` asks for the pixel-major one
-            const uint32_t frow = static_cast<uint32_t>(d->w) * d->c * 4u;
+            const uint32_t frow = static_cast<uint32_t>(d->w) * d->c * static_cast<uint32_t>(qx->esz);
             const Choice c = current_choice(d);
             const bool cm_first = c.kernel != QC_KERNEL_HALO;
             if ((cm_first && make_halo_plan(&ex.e, ex.g, &qx->pl, frow, true)) ||
@@ -1348,7 +1350,8 @@ qc_status launch_fused_stem(QExec &qx, const void *x, float in_scale, const void
     p.f_c = d->c;
     p.f_pad_h = d->pad_h;
     p.f_pad_w = d->pad_w;
-    p.f_rowbytes = d->w * d->c * 4;
+    p.f_rowbytes = d->w * d->c * qx.esz;
+    p.bf16 = qx.esz == 2 ? 1 : 0;
     p.fd_pq = qc::make_fastdiv(static_cast<uint32_t>(p.PQ));
     p.fd_q = qc::make_fastdiv(static_cast<uint32_t>(p.Q));
     p.fd_ntn = qc::make_fastdiv(static_cast<uint32_t>(p.n_tiles_n));
@@ -1364,7 +1367,7 @@ qc_status launch_fused_stem(QExec &qx, const void *x, float in_scale, const void
         // long contiguous TMA row (a 16-byte inner box would cost one request per 16 bytes);
         // rows outside the image are zero-filled (= +0.0f, which quantizes to the zero point)
         const Driver &drv = driver();
-        const cuuint64_t rowb = static_cast<cuuint64_t>(d->w) * d->c * 4;
+        const cuuint64_t rowb = static_cast<cuuint64_t>(d->w) * d->c * qx.esz;
         cuuint64_t k = (rowb + 2047) / 2048;
         while (rowb % (8 * k)) ++k;
         const cuuint64_t piece = rowb / (8 * k);

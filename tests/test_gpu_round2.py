@@ -337,12 +337,14 @@ def test_autotune_records_an_exact_plan():
 
 
 @pytest.mark.parametrize("bits", [8, 4])
-@pytest.mark.parametrize("n_img,relu", [(2, True), (1, False), (5, True)])
+@pytest.mark.parametrize("n_img,relu,bf16", [(2, True, False), (1, False, False), (5, True, False),
+                                             (2, True, True), (3, False, True)])
 @pytest.mark.parametrize("kernel", ["halo_t", "halo"])
-def test_forward_quantize_fused_stem(bits, n_img, relu, kernel):
-    """qconv2d_forward_quantize on the C = 3 stem: one kernel quantizes the fp32 rows (Z4) into
-    its space-to-depth operand tile; compared with oracle quantize (+ a zero-point channel) then
-    the oracle's direct 7x7/s2 conv.  Inputs include NaN, +-inf and exact quantization ties."""
+def test_forward_quantize_fused_stem(bits, n_img, relu, bf16, kernel):
+    """qconv2d_forward_quantize on the C = 3 stem: one kernel quantizes the fp32 (or bf16) rows
+    (Z4) into its space-to-depth operand tile; compared with oracle quantize (+ a zero-point
+    channel) then the oracle's direct 7x7/s2 conv.  Inputs include NaN, +-inf and exact
+    quantization ties (in bf16: the bf16 roundings of them)."""
     cs = ConvShape("stem", n_img, 224, 224, 3, 64, 7, 7, 2, 3)
     rng = np.random.default_rng(60 + bits + n_img)
     xf = float_image(rng, (n_img, 224, 224, 3))
@@ -350,7 +352,13 @@ def test_forward_quantize_fused_stem(bits, n_img, relu, kernel):
     xf.reshape(-1)[:6] = [np.nan, np.inf, -np.inf, 0.5 * s_x, 1.5 * s_x, 2.5 * s_x]
     xt = U4 if bits == 4 else U8
     li = make_layer_inputs(cs, bits, seed=3 + bits, c_store=4, relu=relu, signed_out=not relu)
-    li.x_bytes = oracle.quantize(xf, s_x, 0, xt, c_pad=4)
+    xtensor = torch.from_numpy(xf)
+    if bf16:
+        xtensor = xtensor.to(torch.bfloat16)
+        host = xtensor.view(torch.int16).numpy().view(np.uint16)
+    else:
+        host = xf
+    li.x_bytes = oracle.quantize(host, s_x, 0, xt, c_pad=4, bf16=bf16)
     m, n = oracle.requant_params(li.s_x, li.s_w, li.s_y)
     ref = oracle.conv2d_layer(li, mult=m, shift=n)
     d = qc.make_desc(n_img, 224, 224, 3, 64, 7, 7, stride=2, pad=3, x_t=xt, w_t=S8, y_t=li.y_t,
@@ -363,13 +371,13 @@ def test_forward_quantize_fused_stem(bits, n_img, relu, kernel):
             if prepared:
                 w = qc.qconv_prepare_weights(d, w)
                 d.w_prepared = 1
-                assert qc._lib().qconv2d_quantize_workspace_size(d, qc.QC_F32) == 0   # one kernel
+                assert qc._lib().qconv2d_quantize_workspace_size(d, qc.QC_BF16 if bf16 else qc.QC_F32) == 0   # one kernel
             if kernel == "halo":        # the pixel-major halo, chosen through the plan API
                 qc.qconv_plan_set(d, qc.QC_KERNEL_HALO, 0)
             assert qc.qconv_debug_plan_quantize(d)["kernel"] == want
-            y = qc.qconv2d_forward_quantize(d, torch.from_numpy(xf).to(DEV), s_x, w, b, mm, nn)
+            y = qc.qconv2d_forward_quantize(d, xtensor.to(DEV).contiguous(), s_x, w, b, mm, nn)
             torch.cuda.synchronize()
-            _assert_same(y.cpu().numpy(), ref, f"fused stem {kernel} (prepared={prepared})")
+            _assert_same(y.cpu().numpy(), ref, f"fused stem {kernel} (prepared={prepared}, bf16={bf16})")
     finally:
         qc.qconv_plan_clear()
 
