@@ -301,10 +301,11 @@ class OracleTrunk:
     time: quantize the fp32 stem input, then the 53 layers chained as in Trunk.  Weights and
     scales are regenerated from the same seeds; (m, shift) come from the oracle's R1."""
 
-    def __init__(self, bits: int):
+    def __init__(self, bits: int, stem_dtype: str = "bf16"):
         import oracle
         self.oracle = oracle
         self.bits = bits
+        self.bf16 = stem_dtype == "bf16"   # image() draws the stem input as the bench does
         self.cores = os.cpu_count() or 1
         os.environ.setdefault("OMP_NUM_THREADS", str(self.cores))
         self.x_t = W.U4 if bits == 4 else W.U8
@@ -358,9 +359,12 @@ class OracleTrunk:
     def image(self, layer_subset=None):
         """One random image through quantize + (a subset of) the layers; returns ops done."""
         xf = np.maximum(self.rng.standard_normal((1, 224, 224, 3), dtype=np.float32), 0)
+        if self.bf16:      # round to nearest even bf16 bit patterns (finite inputs)
+            u = xf.view(np.uint32).astype(np.uint64)
+            xf = ((u + 0x7FFF + ((u >> 16) & 1)) >> 16).astype(np.uint16)
         codes = W.post_relu_codes_fast(self.rng, (1, 56, 56, 64), self.bits)
         res2 = (codes[..., 0::2] | (codes[..., 1::2] << 4)).astype(np.uint8) if self.bits == 4 else codes
-        return self.chain(xf, res2, layer_subset)[1]
+        return self.chain(xf, res2, layer_subset, bf16=self.bf16)[1]
 
     def groups(self, n_groups: int):
         tot = sum(self.ops)
@@ -398,9 +402,9 @@ def verify_trunk(trunk: Trunk, images, ot: OracleTrunk = None):
             "bit_exact": not bad, "mismatch": bad[:5], "oracle_s": time.perf_counter() - t0}
 
 
-def oracle_trunk_images_per_s(bits: int, budget_s: float = 15.0, max_images: int = 8):
+def oracle_trunk_images_per_s(bits: int, budget_s: float = 15.0, max_images: int = 8, stem_dtype: str = "bf16"):
     """cpu_baseline leg: whole images through the oracle trunk within a time budget."""
-    ot = OracleTrunk(bits)
+    ot = OracleTrunk(bits, stem_dtype)
     ops_img = sum(ot.ops)
     done_ops = 0
     t0 = time.perf_counter()
@@ -419,7 +423,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
-    ot = OracleTrunk(args.bits)
+    ot = OracleTrunk(args.bits, args.stem_dtype)
     groups = ot.groups(8)
     ops_img = sum(ot.ops)
     for s in range(args.warmup):
@@ -599,7 +603,7 @@ def run_trunk(args):
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        ips, cores, n_img, dt = oracle_trunk_images_per_s(args.bits)
+        ips, cores, n_img, dt = oracle_trunk_images_per_s(args.bits, stem_dtype=args.stem_dtype)
         cpu = {"value": ips, "unit": "images/s", "cores": cores, "kind": "oracle",
                "sample": f"{n_img} image(s) x (quantize + 53 layers), {dt:.1f} s"}
 
