@@ -72,8 +72,42 @@ def chain_pdl():
     return ok
 
 
+def fused_stem(bf16):
+    """qconv2d_forward_quantize on a small C = 3 stem: the channel-major halo kernel quantizes
+    the fp32 / bf16 rows itself (converter warps, code-row ring)."""
+    from workloads import float_image, pack_codes, S8, U8
+    cs = ConvShape("fstem", 1, 64, 64, 3, 64, 7, 7, 2, 3)
+    rng = np.random.default_rng(9)
+    xf = float_image(rng, (1, 64, 64, 3))
+    s_x = 3.0 / 255
+    li = make_layer_inputs(cs, 8, seed=11, c_store=4, relu=True)
+    xt = torch.from_numpy(xf)
+    if bf16:
+        xt = xt.to(torch.bfloat16)
+        host = xt.view(torch.int16).numpy().view(np.uint16)
+    else:
+        host = xf
+    li.x_bytes = oracle.quantize(host, s_x, 0, U8, c_pad=4, bf16=bf16)
+    m, n = oracle.requant_params(li.s_x, li.s_w, li.s_y)
+    ref = oracle.conv2d_layer(li, mult=m, shift=n)
+    d = qc.make_desc(1, 64, 64, 3, 64, 7, 7, stride=2, pad=3, x_t=U8, w_t=S8, y_t=li.y_t,
+                     clamp_lo=li.clamp_lo, clamp_hi=li.clamp_hi)
+    w = torch.from_numpy(np.ascontiguousarray(pack_codes(li.w_codes[..., :3], S8))).to(DEV)
+    b, mm, nn = (torch.from_numpy(a).to(DEV) for a in (li.bias, m, n))
+    y = qc.qconv2d_forward_quantize(d, xt.to(DEV).contiguous(), s_x, w, b, mm, nn)
+    torch.cuda.synchronize()
+    ok = np.array_equal(y.cpu().numpy(), ref)
+    print(f"fused stem ({'bf16' if bf16 else 'fp32'}) {qc.qconv_debug_plan_quantize(d)['kernel_name']} "
+          f"{'ok' if ok else 'MISMATCH'}", flush=True)
+    return ok
+
+
 def main():
     oks = [
+        run(ConvShape("halot8", 2, 14, 14, 64, 64, 3, 3, 1, 1), 8, qc.QC_KERNEL_HALO_T),
+        run(ConvShape("halot4", 2, 14, 14, 64, 64, 3, 3, 1, 1), 4, qc.QC_KERNEL_HALO_T),
+        fused_stem(False),
+        fused_stem(True),
         run(ConvShape("halo8", 2, 14, 14, 64, 64, 3, 3, 1, 1), 8, qc.QC_KERNEL_HALO),
         run(ConvShape("halo4", 2, 14, 14, 64, 64, 3, 3, 1, 1), 4, qc.QC_KERNEL_HALO),
         run(ConvShape("chan8", 2, 8, 16, 64, 128, 1, 1), 8, qc.QC_KERNEL_CHANNEL, 128),
