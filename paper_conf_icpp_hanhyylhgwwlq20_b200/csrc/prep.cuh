@@ -272,39 +272,65 @@ __global__ void __launch_bounds__(256) widen_w4_pad_kernel(const uint8_t *__rest
 
 // int8 KRSC from 4- or 8-bit packed KRSC, rows of c_src channels padded to c_dst with zero
 // weights (A8W4 weights; 8-bit channel padding).
+// rows = K*R*s_dst output filter rows; filter columns s >= s_src and channels c >= c_src are 0.
 __global__ void __launch_bounds__(256) weights_plain_kernel(const uint8_t *__restrict__ w, int8_t *__restrict__ w8,
                                                             int64_t rows, int32_t c_src, int32_t c_dst,
-                                                            int32_t bits, int32_t is_signed) {
+                                                            int32_t bits, int32_t is_signed, int32_t s_src,
+                                                            int32_t s_dst) {
     const int64_t total = rows * c_dst;
     for (int64_t e = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; e < total;
          e += static_cast<int64_t>(gridDim.x) * blockDim.x) {
         const int64_t row = e / c_dst;
         const int32_t c = static_cast<int32_t>(e - row * c_dst);
-        w8[e] = static_cast<int8_t>(c < c_src ? get_code(w, row * c_src + c, bits, is_signed) : 0);
+        const int64_t kr = row / s_dst;
+        const int32_t sc = static_cast<int32_t>(row - kr * s_dst);
+        w8[e] = static_cast<int8_t>(c < c_src && sc < s_src ? get_code(w, (kr * s_src + sc) * c_src + c, bits, is_signed) : 0);
     }
 }
 
 // Activation codes [npix][c_src] -> [npix][c_dst] (same packing), pad channels = zx.
+// One thread = one pixel: its c_src codes, then x_zero codes up to c_dst channels, written as
+// 16-byte vectors (c_dst * bits / 8 is a multiple of 16 for every padded shape qconv.cu makes).
+// npix output pixels of rows w_dst wide; output columns >= w_src are all zx codes.
 __global__ void __launch_bounds__(256) repack_pad_kernel(const uint8_t *__restrict__ x, uint8_t *__restrict__ y,
                                                          int64_t npix, int32_t c_src, int32_t c_dst,
-                                                         int32_t bits, int32_t zx) {
+                                                         int32_t bits, int32_t zx, int32_t w_src, int32_t w_dst) {
     const int32_t ob = c_dst * bits / 8;      // output bytes per pixel
-    const int64_t total = npix * ob;
-    for (int64_t e = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; e < total;
-         e += static_cast<int64_t>(gridDim.x) * blockDim.x) {
-        const int64_t pix = e / ob;
-        const int32_t j = static_cast<int32_t>(e - pix * ob);
-        if (bits == 8) {
-            y[e] = j < c_src ? x[pix * c_src + j] : static_cast<uint8_t>(zx & 0xFF);
-        } else {
-            uint32_t v = 0;
-            for (int h = 0; h < 2; ++h) {
-                const int32_t c = 2 * j + h;
-                const int64_t idx = pix * c_src + c;
-                const uint32_t nib = c < c_src ? ((x[idx >> 1] >> (4 * (idx & 1))) & 0xFu) : (static_cast<uint32_t>(zx) & 0xFu);
-                v |= nib << (4 * h);
+    const uint32_t z8 = static_cast<uint32_t>(zx) & 0xFFu;
+    const uint32_t z4 = static_cast<uint32_t>(zx) & 0xFu;
+    for (int64_t pix = blockIdx.x * static_cast<int64_t>(blockDim.x) + threadIdx.x; pix < npix;
+         pix += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const int64_t row = pix / w_dst;
+        const int32_t col = static_cast<int32_t>(pix - row * w_dst);
+        const int32_t c_in = col < w_src ? c_src : 0;  // codes taken from x (the rest are zx)
+        const int64_t base = (row * w_src + col) * c_src;   // first code of the pixel (element index)
+        uint4 *dst = reinterpret_cast<uint4 *>(y + pix * ob);
+        for (int32_t q = 0; q < ob / 16; ++q) {
+            uint32_t w[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                uint32_t v = 0;
+#pragma unroll
+                for (int b = 0; b < 4; ++b) {
+                    const int32_t j = 16 * q + 4 * k + b;       // output byte
+                    uint32_t byte;
+                    if (bits == 8) {
+                        byte = j < c_in ? static_cast<uint32_t>(__ldg(x + base + j)) : z8;
+                    } else {
+                        byte = 0;
+#pragma unroll
+                        for (int h = 0; h < 2; ++h) {
+                            const int32_t c = 2 * j + h;
+                            const int64_t idx = base + c;
+                            const uint32_t nib = c < c_in ? ((static_cast<uint32_t>(__ldg(x + (idx >> 1))) >> (4 * (idx & 1))) & 0xFu) : z4;
+                            byte |= nib << (4 * h);
+                        }
+                    }
+                    v |= byte << (8 * b);
+                }
+                w[k] = v;
             }
-            y[e] = static_cast<uint8_t>(v);
+            dst[q] = make_uint4(w[0], w[1], w[2], w[3]);
         }
     }
 }

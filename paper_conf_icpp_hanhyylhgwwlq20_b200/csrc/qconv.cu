@@ -247,6 +247,7 @@ struct Exec {
     bool zx, zw;
     size_t off_w, off_x, off_zx, off_cs, off_x1, ws_total;
     int prologue;         // qconv_plan.prologue mask
+    int s_pad;            // XF_PAD: extra zero-weight filter columns (odd S -> even: halo tap pairs)
 };
 
 int32_t s2d_channels(int32_t c) {
@@ -272,6 +273,8 @@ qconv_desc s2d_of(const qconv_desc *d, const Geometry &g) {
     return o;
 }
 
+bool halo_eligible(const qconv_desc *e, const Geometry &g);   // after make_halo_plan below
+
 qc_status derive_exec(const qconv_desc *d, bool allow_float, Exec *ex) {
     qc_status s = validate_desc(d, &ex->gu, allow_float);
     if (s != QC_OK) return s;
@@ -292,6 +295,26 @@ qc_status derive_exec(const qconv_desc *d, bool allow_float, Exec *ex) {
     } else {
         ex->xform = XF_PAD;
         ex->e.c = (xbits == 8 && d->c < 16) ? 16 : (d->c + 31) / 32 * 32;
+    }
+    ex->s_pad = 0;
+    if (ex->xform == XF_PAD && ex->e.c == 16 && xbits == 8 && (d->s % 2) && d->stride_w == 1 &&
+        d->stride_h == 1 && d->dil_h == 1 && d->dil_w == 1 && d->x_zero == 0 && d->w_zero == nullptr) {
+        // C = 16 byte codes pair two filter taps per K = 32 MMA in the halo kernels, which need
+        // an even S: one more filter column of zero weights, one more input column of zero-point
+        // codes (the column it would read past the image) -- same products, same P and Q --
+        // taken only when a halo plan then exists (the im2col path would just do 1/S more MMAs)
+        qconv_desc e2 = ex->e;
+        e2.s += 1;
+        e2.w += 1;
+        e2.x_t = byte_container(d->x_t);
+        e2.w_t = byte_container(d->w_t);
+        Geometry g2;
+        if (validate_desc(&e2, &g2, allow_float) == QC_OK && g2.P == ex->gu.P && g2.Q == ex->gu.Q &&
+            halo_eligible(&e2, g2)) {
+            ex->e.s = e2.s;
+            ex->e.w = e2.w;
+            ex->s_pad = 1;
+        }
     }
     qconv_desc &e = ex->e;
     if (ex->xform == XF_S2D) ex->wprep = WP_S2D;
@@ -360,10 +383,11 @@ qc_status prepare_weights_exec(const Exec &ex, const void *w, void *out, cudaStr
             break;
         }
         case WP_PLAIN: {
-            const int64_t total = rows * e.c;
+            const int64_t rows_e = static_cast<int64_t>(e.k) * e.r * e.s;
+            const int64_t total = rows_e * e.c;
             const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, 4096));
             qc::weights_plain_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(w), static_cast<int8_t *>(out),
-                                                           rows, d->c, e.c, dtype_bits(d->w_t), sgn);
+                                                           rows_e, d->c, e.c, dtype_bits(d->w_t), sgn, d->s, e.s);
             break;
         }
         case WP_S2D: {
@@ -787,6 +811,11 @@ bool make_halo_plan(const qconv_desc *d, const Geometry &g, Plan *pl, uint32_t f
     return true;
 }
 
+bool halo_eligible(const qconv_desc *e, const Geometry &g) {
+    Plan tmp;
+    return make_halo_plan(e, g, &tmp, 0, true) || make_halo_plan(e, g, &tmp, 0, false);
+}
+
 qc_status encode_halo_maps(const qconv_desc *d, const Geometry &g, const qc::ConvParams &p,
                            const void *x, const void *w8, void *y, CUtensorMap *hm, CUtensorMap *bm,
                            CUtensorMap *ym, bool cm = false) {
@@ -1076,10 +1105,10 @@ qc_status run_prologue(const Exec &ex, const void *x, const void *w, void *ws, c
         *x_e = wsb + ex.off_x;
     } else if (ex.xform == XF_PAD) {
         const int64_t npix = static_cast<int64_t>(d->n) * d->h * d->w;
-        const int64_t total = npix * ex.g.c_bytes;
-        const int grid = static_cast<int>(std::min<int64_t>((total + 255) / 256, static_cast<int64_t>(num_sms()) * 16));
-        qc::repack_pad_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(x), wsb + ex.off_x, npix, d->c,
-                                                    e.c, dtype_bits(d->x_t), d->x_zero);
+        const int grid = static_cast<int>(std::min<int64_t>((npix + 255) / 256, static_cast<int64_t>(num_sms()) * 16));
+        const int64_t npix_e = static_cast<int64_t>(e.n) * e.h * e.w;
+        qc::repack_pad_kernel<<<grid, 256, 0, st>>>(static_cast<const uint8_t *>(x), wsb + ex.off_x, npix_e, d->c,
+                                                    e.c, dtype_bits(d->x_t), d->x_zero, d->w, e.w);
         *x_e = wsb + ex.off_x;
     }
     if (ex.zx) {

@@ -287,13 +287,33 @@ def test_channel_padding(cs, bits):
 
 
 def test_vgg16_conv1_1_batch2():
-    """VGG-16 conv1_1 (C = 3, 3x3/s1, 224x224), the layer round 1 could not run."""
+    """VGG-16 conv1_1 (C = 3, 3x3/s1, 224x224), the layer round 1 could not run.  Its codes are
+    padded to 16 channels and its filter to 3x4 (a zero-weight column, one zero-point input
+    column) so the channel-major halo kernel pairs its taps -- checked to be the plan taken."""
     cs = vgg16_convs(2)[0]
     li = make_layer_inputs(cs, 8, seed=3000)
     m, n = oracle.requant_params(li.s_x, li.s_w, li.s_y)
     ref = oracle.conv2d_layer(li, mult=m, shift=n)
-    got, _ = _gpu(li, m, n)
+    got, plan = _gpu(li, m, n)
+    assert plan["kernel_name"] == "halo_t", plan
     _assert_same(got, ref, "vgg conv1_1")
+
+
+@pytest.mark.parametrize("cs", [
+    ConvShape("c3s5", 2, 20, 23, 3, 32, 5, 5, 1, 2),        # odd S = 5 -> 6, pixel-major halo
+    ConvShape("c7s3", 3, 16, 29, 7, 64, 3, 3, 1, 1),        # K = 64 -> channel-major halo
+    ConvShape("c1s1x3", 2, 12, 40, 1, 64, 1, 3, 1, 0),      # 1x3 filter, no padding
+], ids=lambda v: v.name)
+def test_odd_filter_width_tap_pairs(cs):
+    """8-bit, C < 16, stride 1, odd S: the filter gains a zero-weight column and the input a
+    zero-point column (same products, same P x Q) so a halo kernel can pair taps."""
+    li = make_layer_inputs(cs, 8, seed=cs.c * 13 + cs.s, relu=True)
+    m, n = oracle.requant_params(li.s_x, li.s_w, li.s_y)
+    ref = oracle.conv2d_layer(li, mult=m, shift=n)
+    for prepared in (False, True):
+        got, plan = _gpu(li, m, n, prepared=prepared)
+        assert plan["kernel_name"] in ("halo", "halo_t"), plan
+        _assert_same(got, ref, f"{cs.name} prepared={prepared}")
 
 
 TUNE_SHAPES = [ConvShape("t3", 4, 14, 14, 128, 128, 3, 3, 1, 1),
