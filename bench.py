@@ -631,9 +631,9 @@ def run_trunk(args):
                        "global_batch": global_batch, "per_gpu_batch": per_gpu,
                        "layers": len(trunk.layers), "parallelism": f"dp{world} (batch shards)",
                        "stem_input": f"{trunk.stem_dtype} NHWC image, quantized inside the stem kernel",
-                       "l2": f"inputs > L2: {trunk.x_float.numel() * trunk.x_float.element_size() / 1e6:.0f} MB "
-                             f"{trunk.stem_dtype} stem input and ~2.4 GB of trunk traffic per step "
-                             "(at 256 images per GPU)",
+                       "l2": f"working set > L2: ~2.4 GB of trunk traffic per step (at 256 images per GPU) "
+                             f"streams through the 126 MB L2, evicting the {trunk.x_float.numel() * trunk.x_float.element_size() / 1e6:.0f} MB "
+                             f"{trunk.stem_dtype} stem input before the next step reads it",
                        "graph": "one CUDA graph per step (PDL between the conv kernels), replayed",
                        "plans": plans_note},
             "tops": trunk.ops_per_step / (ms_per_step / 1e3) / 1e12,
