@@ -57,7 +57,7 @@ int main() {
     long long *out; cudaMalloc(&out, 148 * 8);
     int *sink; cudaMalloc(&sink, 64);
     const char *names[] = {"IMAD.HI(+64b)", "SHF(funnel)", "I2IP.U4.SAT", "IMAD", "IADD", "LOP3", "PRMT", "FFMA", "SHR.S32", "IMNMX+IADD", "mad.hi.s32", "mul.hi.u32", "mul.wide.lo", "mad.wide", "I2F+FADD", "F2I.floor+..", "wide>>40", "DFMA", "DADD.RD", "I2F.F64"};
-    for (int op = 17; op < 20; ++op)
+    for (int op = 0; op < 20; ++op)
         for (int warps : {4, 8, 16}) {
             const int iters = 2048;
             for (int rep = 0; rep < 2; ++rep) {
